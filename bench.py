@@ -1,0 +1,316 @@
+"""pgvc benchmark — VC instances checked per second (BASELINE.json metric).
+
+Workload (N=1 headline, BASELINE.json configs[1] = C2): CUDA SDK reduction variants
+reduce0..reduce6 checked pairwise against reduce0 plus the injected off-by-one pair
+(reduce2 vs reduce2_obo); B = 2^0..2^10 elements per block, N = B..2^16, 64 seeds
+per GPU (RAND32), checks EQUIV|RACE|OOB.  One step = every pair over the whole
+space: input generation (K1), both evaluation kernels (K2), comparison (K3),
+compaction (K4) and the H9 all_reduce of the first-counterexample key (MIN) and
+the counts (SUM).  Multi-GPU: every rank checks its own 64 seeds (seed_base =
+rank * 64), i.e. weak scaling; the only collective is H9.
+
+`--impl reference` times the CPU oracle (oracle/, test infrastructure) on the
+host cores on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "VC instances checked/sec (n x tid x round x seed)"
+UNIT = "instances/s"
+SEEDS_PER_GPU = 64
+# SURVEY.md §8(d) algorithmic work per instance (thread x round) of a reduction round:
+# ~10 integer IR ops + 2 shared loads + 1 shared store = 13 ops.
+OPS_PER_INSTANCE = 13
+SM_COUNT = 148
+ALU_LANES_PER_SM_CLK = 64   # IADD3/LOP3 alu pipe: 4 SMSP x 16 lanes/clk (B300_MICROARCH: rt_SMSP = 2)
+
+
+def workload_desc():
+    return ("C2: SDK reduce0 vs reduce1..6 + reduce2 vs reduce2_obo, B=2^0..2^10, N=B..2^16, "
+            "%d RAND32 seeds per GPU, checks EQUIV|RACE|OOB" % SEEDS_PER_GPU)
+
+
+def c2_pairs():
+    from paper_conf_ipps_lig12_b200 import workloads as W
+    return W.c2(n_seeds=SEEDS_PER_GPU)
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+        self.thread = None
+
+    def start(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + q,
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.proc = None
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 7:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        if self.thread:
+            self.thread.join(timeout=2)
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return json.load(f)
+    except OSError:
+        return {}
+
+
+def ncu_traffic():
+    """Per-launch DRAM bytes of the evaluation kernel from the committed ncu capture (or None)."""
+    p = os.path.join(ROOT, "profiles", "k2_traffic.json")
+    try:
+        with open(p) as f:
+            return json.load(f).get("bytes_per_launch")
+    except (OSError, ValueError):
+        return None
+
+
+# ---------------------------------------------------------------- CPU oracle (reference arm / cpu_baseline)
+def _oracle_shard(args):
+    rank, world, pts_max_log_n, n_seeds = args
+    sys.path.insert(0, ROOT)
+    import oracle
+    from paper_conf_ipps_lig12_b200 import workloads as W
+    inst = 0
+    for w in W.c2(n_seeds=n_seeds, max_log_n=pts_max_log_n, max_log_b=10):
+        r = oracle.check(W.subject(w.src), W.subject(w.tgt), w.launch_src, w.launch_tgt, n_seeds=n_seeds,
+                         rank=rank, world=world, checks=w.checks, cap=1 << 16)
+        inst += r["counts"][0]
+    return inst
+
+
+def oracle_sample(max_log_n=12, n_seeds=4):
+    """The oracle as it stands, one process per host core over seed shards, on the
+    C2 pairs restricted to N <= 2^max_log_n and n_seeds seeds."""
+    import multiprocessing as mp
+    sys.path.insert(0, ROOT)
+    import oracle
+    oracle.build()
+    cores = len(os.sched_getaffinity(0))
+    world = min(cores, n_seeds)
+    t0 = time.perf_counter()
+    with mp.get_context("fork").Pool(world) as pool:
+        inst = sum(pool.map(_oracle_shard, [(r, world, max_log_n, n_seeds) for r in range(world)]))
+    dt = time.perf_counter() - t0
+    sample = ("C2 pairs restricted to N <= 2^%d (B = 2^0..2^10), seeds 0..%d, %d processes"
+              % (max_log_n, n_seeds - 1, world))
+    return inst, dt, world, sample
+
+
+def run_reference(args):
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return
+    inst_total, t_total = 0, 0.0
+    for _ in range(args.warmup):
+        oracle_sample(max_log_n=args.ref_log_n, n_seeds=args.ref_seeds)
+    for _ in range(args.steps):
+        inst, dt, cores, sample = oracle_sample(max_log_n=args.ref_log_n, n_seeds=args.ref_seeds)
+        inst_total += inst
+        t_total += dt
+    v = inst_total / t_total
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * t_total / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": workload_desc(), "sample": sample},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- GPU arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="pgvc", choices=["pgvc", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--ref-log-n", type=int, default=12)
+    ap.add_argument("--ref-seeds", type=int, default=4)
+    args = ap.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+
+    import torch
+    import torch.distributed as dist
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    from paper_conf_ipps_lig12_b200 import build, pgvc
+    if rank == 0 or world == 1:
+        build.build()
+    if world > 1:
+        dist.barrier()
+    wls = c2_pairs()
+    irs = {}
+    for w in wls:
+        for name in (w.src, w.tgt):
+            if name not in irs:
+                from paper_conf_ipps_lig12_b200 import workloads as W
+                irs[name] = pgvc.load_ir(W.subject(name))
+    stream = torch.cuda.Stream()
+    first_key = torch.empty(11, dtype=torch.int64, device="cuda")
+    counts = torch.empty(16, dtype=torch.int64, device="cuda")
+    step_keys = torch.empty(11, dtype=torch.int64, device="cuda")
+    step_counts = torch.zeros(16, dtype=torch.int64, device="cuda")
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+
+    def step():
+        """One pass of the whole path over the workload; returns (instances, runs)."""
+        runs = []
+        with torch.cuda.stream(stream):
+            step_keys.fill_(2 ** 63 - 1)
+            step_counts.zero_()
+            for w in wls:
+                sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=w.n_seeds, seed_base=rank * SEEDS_PER_GPU,
+                                checks=w.checks, stream=stream.cuda_stream, first_key=first_key, counts=counts)
+                runs.append(pgvc.check_equiv(irs[w.src], irs[w.tgt], sp))
+                torch.minimum(step_keys, first_key, out=step_keys)
+                step_counts.add_(counts)
+            if world > 1:   # H9: the only cross-GPU traffic
+                dist.all_reduce(step_keys, op=dist.ReduceOp.MIN)
+                dist.all_reduce(step_counts, op=dist.ReduceOp.SUM)
+        return runs
+
+    def collect(runs):
+        d2h = 0
+        recs_total = 0
+        for r in runs:
+            recs, s = r.collect(cap=1 << 16)
+            recs_total += len(recs)
+            d2h += 64 * len(recs) + 8 * (16 + 11)
+        return d2h, recs_total
+
+    # warm-up (also JIT-compiles every evaluation kernel variant)
+    for _ in range(max(3, args.warmup)):
+        collect(step())
+    torch.cuda.synchronize()
+
+    clocks = Clocks(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    dev_ms, wall_s, inst_local, launches, h2d, d2h, eval_ms, n_k2, k2_inst = 0.0, 0.0, 0, 0, 0, 0, 0.0, 0, 0
+    for _ in range(args.steps):
+        flush.fill_(1)                       # L2 flush between timed steps (not timed)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0 = time.perf_counter()
+        e0.record(stream)
+        runs = step()
+        e1.record(stream)
+        dd, _ = collect(runs)                # records D2H (end-to-end result read)
+        wall_s += time.perf_counter() - t0
+        stream.synchronize()
+        dev_ms += e0.elapsed_time(e1)
+        d2h += dd
+        for r in runs:
+            t = r.timing()
+            launches += t["launches"]
+            h2d += t["h2d_bytes"]
+            eval_ms += t["ms_eval"]
+        inst_local += int(step_counts[0].item()) if world == 1 else 0
+        if world > 1:
+            inst_local += int(step_counts[0].item())   # already all-reduced: whole-job instances
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    t = torch.tensor([dev_ms, wall_s], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    dev_ms, wall_s = float(t[0]), float(t[1])
+    inst_total = inst_local  # whole job (all ranks) per the all-reduced counts
+    value = inst_total / (dev_ms / 1000.0)
+    e2e = inst_total / wall_s
+    peaks = measured_peaks()
+    sm_max = clk.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
+    alu_peak = SM_COUNT * ALU_LANES_PER_SM_CLK * sm_max * 1e6
+    per_gpu_inst = inst_total / world
+    achieved_ops = per_gpu_inst * OPS_PER_INSTANCE / (eval_ms / 1000.0) if eval_ms else None
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": workload_desc(), "seeds_per_gpu": SEEDS_PER_GPU, "l2": "flushed between steps",
+                   "parallelism": "dp%d over seeds" % world},
+        "roofline": {"bound": "alu", "achieved": achieved_ops / 1e12 if achieved_ops else None,
+                     "peak": alu_peak / 1e12, "unit": "Tops/s (int32, algorithmic IR ops)",
+                     "frac": (achieved_ops / alu_peak) if achieved_ops else None, "traffic": ncu_traffic(),
+                     "kernel": "pgk_eval (K2)", "ops_per_instance": OPS_PER_INSTANCE,
+                     "k2_ms_per_step": eval_ms / args.steps,
+                     "peak_source": "148 SM x 64 int32 lanes/clk x sm_max_mhz (DESIGN.md §6)"},
+        "e2e": {"value": e2e, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
+                "d2h_bytes_per_step": d2h // args.steps},
+        "gpu_launches": launches // args.steps * args.steps,
+        "clocks": clk,
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        inst, dt, cores, sample = oracle_sample()
+        line["cpu_baseline"] = {"value": inst / dt, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,160 @@
+/*
+ * pgvc.h — C ABI of libpgvc.so: bounded, exhaustive instantiation of PUGpara's
+ * parameterized verification conditions on a B200.
+ *
+ * Paper: G. Li, G. Gopalakrishnan, "Parameterized Verification of GPU Kernel
+ * Programs" (/root/reference/PAPER.md, cited Lnnn).  Semantics readings X1-X21
+ * are in DESIGN.md §2.
+ *
+ * Conventions
+ *   - Every function returns a PG_* status (0 = success); no C++ exception
+ *     crosses this boundary.  pg_last_error() returns a thread-local message
+ *     ("line:col: ..." for parse/type errors), valid until the next call on the
+ *     same thread.
+ *   - Handles (pg_ir, pg_run) are owned by the caller and freed with
+ *     pg_ir_free / pg_run_free.  A pg_run owns its device and host buffers.
+ *   - Pointers in pg_space are borrowed for the duration of the call, except
+ *     d_first_key / d_counts / cuda_stream, which are borrowed (owned by the
+ *     caller, e.g. torch) until pg_collect_cex returns.
+ *   - pg_check_* only ENQUEUE work on cuda_stream; pg_collect_cex synchronises
+ *     that stream.  No collective is issued by the library: the caller may
+ *     all_reduce d_first_key (MIN) and d_counts (SUM) between pg_check_* and
+ *     pg_collect_cex (H9).
+ *   - There is no CPU fallback: without a usable CUDA device every check
+ *     returns PG_E_CUDA.
+ */
+#ifndef PGVC_H
+#define PGVC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct pg_ir pg_ir;    /* one loaded kernel: parsed, checked, code-generated; immutable */
+typedef struct pg_run pg_run;  /* result set of one check */
+
+enum {
+    PG_OK = 0,
+    PG_E_ARG = -1,    /* bad argument */
+    PG_E_PARSE = -2,  /* syntax error in the kernel text (line:col in pg_last_error) */
+    PG_E_TYPE = -3,   /* semantic error: undeclared name, sync under thread-dependent control (X18), ... */
+    PG_E_LIMIT = -4,  /* static or launch limit exceeded (arrays > 2^24 words, > 4096 threads/block, ...) */
+    PG_E_CUDA = -5,   /* CUDA driver / runtime / NVRTC failure, or no device */
+    PG_E_OOM = -6,    /* device allocation failed */
+    PG_E_STATE = -7   /* call out of order (e.g. collect on a run that was never checked) */
+};
+
+enum { PG_IN_RAND32 = 0, PG_IN_BITS01 = 1, PG_IN_RANGE = 2 };                 /* X8 */
+enum { PG_CHK_EQUIV = 1, PG_CHK_RACE = 2, PG_CHK_OOB = 4, PG_CHK_BANK = 8, PG_CHK_COALESCE = 16 };
+enum { PG_BANKS_32 = 0, PG_BANKS_16_HALFWARP = 1 };                             /* X9 */
+enum {                                                                          /* X17 */
+    PG_CEX_BARRIER_DIV = 0, PG_CEX_OOB = 1, PG_CEX_RACE_WW = 2, PG_CEX_RACE_RW = 3, PG_CEX_RACE_XB = 4,
+    PG_CEX_MISMATCH = 5, PG_CEX_BANK = 6, PG_CEX_UNCOALESCED = 7, PG_CEX_UNINIT = 8, PG_CEX_LIMIT = 9,
+    PG_N_KINDS = 10
+};
+
+/* One value of the paper's parameter n (L110-L116): grid and block shape plus
+ * the kernel's scalar parameters in declaration order. */
+typedef struct {
+    uint32_t gdim[3], bdim[3];
+    int32_t scalar[8];
+    uint32_t n_scalar;
+} pg_launch;
+
+/* The bounded parameter space of one check (H1).  launch_src[i] and
+ * launch_tgt[i] describe the same point n for the two kernels (the target may
+ * use another block shape, e.g. reduce3 uses bdim = B/2); index order is the
+ * witness order (X16).  Seeds seed_base + j for j in [0, n_seeds); this call
+ * covers the shard j = rank, rank + world, ... */
+typedef struct {
+    const pg_launch *launch_src, *launch_tgt;  /* launch_tgt may be NULL (= launch_src) */
+    uint32_t n_launch;                         /* < 2^18 */
+    uint64_t seed_base;
+    uint32_t n_seeds;                          /* < 2^24 */
+    uint32_t input_mode, input_range;          /* PG_IN_*, k for PG_IN_RANGE */
+    uint32_t bits;                             /* arithmetic width w (X2): 1..32, default 32 */
+    uint32_t checks, bank_model, max_cex;      /* PG_CHK_* mask; PG_BANKS_*; max records kept */
+    int32_t rank, world;                       /* shard of (launch, seed) instances */
+    void *cuda_stream;                         /* borrowed cudaStream_t (0 = legacy default stream) */
+    int64_t *d_first_key;                      /* borrowed device int64[11]: [0] min failing key, [1+k] min key of kind k; INT64_MAX = none */
+    int64_t *d_counts;                         /* borrowed device int64[16]: [0] instances (X19), [1+k] events of kind k,
+                                                  [11] records, [12] failing (launch, seed) instances */
+} pg_space;
+
+/* One counterexample record (X16): the minimum event of its (launch, seed,
+ * kernel, kind) slot, and the slot's event count.  tid_a/tid_b are global
+ * linear thread ids (XB: block ids). */
+typedef struct {
+    uint64_t key, count;
+    uint32_t kind, launch, seed_idx, kernel, round, site, array, addr, tid_a, tid_b, val_a, val_b;
+} pg_cex;
+
+typedef struct {
+    uint64_t instances;        /* X19 */
+    uint64_t n_fail;           /* failing (launch, seed) instances */
+    uint64_t n_records;
+    int64_t first_key;         /* min failing key (INT64_MAX: none) */
+    uint32_t first_launch;     /* launch index of first_key (0xFFFFFFFF: none) = first-witness n */
+    uint32_t first_seed_idx;
+    uint64_t per_kind[PG_N_KINDS];
+    int64_t first_key_kind[PG_N_KINDS];
+} pg_summary;
+
+/* Parse, check and code-generate one kernel (the IR of DESIGN.md §4; the
+ * paper's C subset, L122-L171).  `text` need not be NUL-terminated.
+ * Errors: PG_E_PARSE / PG_E_TYPE with line:col, PG_E_LIMIT. */
+int pg_load_ir(const char *text, size_t len, pg_ir **out);
+
+/* Comparative assertion (L438-L444, L652-L657): both kernels on every launch
+ * and seed of the space, same initial global arrays (X7), compare every array
+ * that is out/inout in either kernel; plus the checks selected in sp->checks
+ * (RACE: WW/RW/XB; OOB: out-of-bounds and uninitialised reads; BANK/COALESCE
+ * report-only).  Enqueues on sp->cuda_stream. */
+int pg_check_equiv(const pg_ir *src, const pg_ir *tgt, const pg_space *sp, pg_run **out);
+
+/* Race premise of the key observation (L516-L520, L660-L662) for one kernel:
+ * WW / RW / XB / OOB (and LIMIT) over the space; checks = RACE|OOB regardless
+ * of sp->checks. */
+int pg_check_races(const pg_ir *k, const pg_space *sp, pg_run **out);
+
+/* Bank-conflict and coalescing conditions (L21-L24, L146-L150; X9) for one
+ * kernel; BANK / UNCOALESCED records are failing in this mode.  Per-site
+ * statistics are retrievable with pg_collect_site_stats. */
+int pg_check_banks(const pg_ir *k, const pg_space *sp, pg_run **out);
+
+/* Synchronise the run's stream, copy up to `cap` records (canonical key
+ * order) into buf, report how many exist in *n_written (may exceed cap), and
+ * fill *sum (may be NULL) from d_first_key / d_counts as they are now. */
+int pg_collect_cex(pg_run *r, pg_cex *buf, size_t cap, size_t *n_written, pg_summary *sum);
+
+/* Per-site bank/coalescing statistics of a run: uint64
+ * [n_launch][2 kernels][max_sites][8] = [space (1 shared, 2 global), warp
+ * accesses, conflicted|uncoalesced, max degree|sectors, sum degree|sectors,
+ * sum ideal, sum active lanes, 0]; sites >= max_sites are dropped. */
+int pg_collect_site_stats(pg_run *r, uint64_t *buf, uint32_t max_sites);
+
+/* Introspection of a loaded kernel. */
+int pg_ir_info(const pg_ir *k, uint32_t *n_sites, uint32_t *n_globals, uint32_t *n_scalars);
+/* Generated CUDA source of the evaluation kernel for (bits, checks, bank_model). */
+int pg_ir_source(const pg_ir *k, uint32_t bits, uint32_t checks, uint32_t bank_model, char *buf, size_t cap,
+                 size_t *len);
+/* Compile the evaluation kernel variant now (NVRTC -> sm_100a cubin); no GPU needed. */
+int pg_ir_compile(const pg_ir *k, uint32_t bits, uint32_t checks, uint32_t bank_model);
+
+/* Device time of the run's evaluation kernels and of the whole check (CUDA
+ * events on the run's stream, ms), the number of CUDA kernels it launched and
+ * the host->device bytes it copied (launch tables, work lists). */
+int pg_run_timing(pg_run *r, float *ms_eval, float *ms_total, uint32_t *n_launches, uint64_t *h2d_bytes);
+
+const char *pg_last_error(void);
+void pg_ir_free(pg_ir *k);
+void pg_run_free(pg_run *r);
+const char *pg_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PGVC_H */

@@ -1,0 +1,407 @@
+// codegen.cpp — IR -> CUDA C++ of the evaluation kernel (K2).
+//
+// The kernel body becomes a re-entrant "segment" function: each call runs one
+// emulated thread from its resume point to the next barrier (`return k`) or to
+// the end (`return PG_END`); the runtime (device_rt.cuh) performs the round
+// protocol between calls.  Control flow follows the uniformity analysis:
+//   * block-uniform if / loop  -> real branches (gotos at function top level,
+//     so a barrier inside a uniform loop is simply a resume label);
+//   * thread-dependent if / loop -> if-converted with per-lane predicates
+//     and warp-uniform `__any_sync` skips, so every lane of a warp executes
+//     every access site together (the lock-step warp access of X9) and the
+//     warp-level bank / coalescing intrinsics see the whole warp.
+// Loads are predicated (short-circuit && || ?: keep their guards, X2/X21).
+#include <cstdio>
+#include <sstream>
+
+#include "front.hpp"
+
+namespace pgf {
+
+namespace {
+
+std::string hex(uint32_t v) {
+    char b[16];
+    std::snprintf(b, sizeof b, "0x%08xu", v);
+    return b;
+}
+
+struct Gen {
+    const Kernel& K;
+    const CodegenOptions& O;
+    uint32_t mask;
+    std::ostringstream body;
+    int ntmp = 0, nlabel = 0, nsync = 0;
+
+    struct Loop {
+        int id;
+        bool uniform;
+        std::string act;      // non-uniform: active-lane predicate
+        size_t body_depth;    // non-uniform: predicate-stack index of the body predicate
+        int cont_label = -1, exit_label = -1;
+    };
+    std::vector<std::string> preds;  // thread-dependent predicate variables, innermost last
+    std::vector<Loop> loops;
+
+    Gen(const Kernel& k, const CodegenOptions& o) : K(k), O(o) {
+        mask = o.bits >= 32 ? 0xFFFFFFFFu : ((1u << o.bits) - 1u);
+    }
+
+    std::string tmp(const char* p = "t") { return std::string("_") + p + std::to_string(ntmp++); }
+    int label() { return nlabel++; }
+    void line(const std::string& s) { body << "  " << s << "\n"; }
+    bool uniform_ctx() const { return preds.empty(); }
+    std::string cur() const { return preds.empty() ? std::string("1u") : preds.back(); }
+    std::string eff() const { return preds.empty() ? std::string("t.live") : "(" + preds.back() + " & t.live)"; }
+
+    bool reader_tracked(int arr) const {
+        const ArrayDecl& a = K.arrays[(size_t)arr];
+        return (O.checks & PG_RACE_BIT) && a.written && a.read && a.space != PRIVATE;
+    }
+    static constexpr uint32_t PG_RACE_BIT = 2;
+
+    uint32_t priv_size(const ArrayDecl& a) const {
+        uint64_t s = 1;
+        for (const Node* d : a.dims) s *= d->lit;
+        return (uint32_t)s;
+    }
+
+    // ---------------------------------------------------------------- expressions
+    std::string flat_index(const Node* n, int arr, const std::string& pr) {
+        std::vector<std::string> iv;
+        for (const Node* k : n->kids) iv.push_back(ex(k, pr));
+        const ArrayDecl& a = K.arrays[(size_t)arr];
+        std::string f = tmp("f");
+        line("u32 " + f + " = " + iv[0] + ";");
+        for (size_t k = 1; k < iv.size(); k++) {
+            std::string dim;
+            if (a.space == PRIVATE) dim = hex(a.dims[k]->lit);
+            else dim = "C.L->arr[" + std::to_string(arr) + "].d" + std::to_string(k);
+            line(f + " = " + f + " * " + dim + " + " + iv[k] + ";");
+        }
+        return f;
+    }
+    std::string ex(const Node* n, const std::string& pr) {
+        switch (n->kind) {
+        case NK::Lit: return hex(n->lit & mask);
+        case NK::Var: return "F.v" + std::to_string(n->ref);
+        case NK::Builtin: {
+            int c = n->ref % 3;
+            std::string src;
+            if (n->ref < 3) src = "t.tid[" + std::to_string(c) + "]";
+            else if (n->ref < 6) src = "C.bid[" + std::to_string(c) + "]";
+            else if (n->ref < 9) src = "C.L->bdim[" + std::to_string(c) + "]";
+            else src = "C.L->gdim[" + std::to_string(c) + "]";
+            return "pg_m(" + src + ")";
+        }
+        case NK::Elem: {
+            const ArrayDecl& a = K.arrays[(size_t)n->ref];
+            std::string f = flat_index(n, n->ref, pr);
+            std::string r = tmp();
+            std::string A = std::to_string(n->ref), S = std::to_string(n->site) + "u";
+            if (a.space == SHARED) {
+                line("u32 " + r + " = pg_ld_sh<" + A + ", " + (reader_tracked(n->ref) ? "true" : "false") +
+                     ">(C, t, ss, " + pr + ", " + f + ", " + S + ");");
+            } else if (a.space == GLOBAL) {
+                if (a.written)
+                    line("u32 " + r + " = pg_ld_gt<" + A + ", " + (reader_tracked(n->ref) ? "true" : "false") +
+                         ">(C, t, ss, " + pr + ", " + f + ", " + S + ");");
+                else
+                    line("u32 " + r + " = pg_ld_gi<" + A + ">(C, t, ss, " + pr + ", " + f + ", " + S + ");");
+            } else {
+                line("u32 " + r + " = pg_priv_ok(C, t, " + pr + ", " + f + ", " + hex(priv_size(a)) + ", " +
+                     hex(0x200u + (uint32_t)a.slot) + ", " + S + ", 0u, 0u) ? F.p" + std::to_string(a.slot) + "[" +
+                     f + "] : 0u;");
+            }
+            return r;
+        }
+        case NK::Neg: return def("pg_neg(" + ex(n->kids[0], pr) + ")");
+        case NK::BitNot: return def("pg_not(" + ex(n->kids[0], pr) + ")");
+        case NK::LogNot: return def("(u32)(" + ex(n->kids[0], pr) + " == 0u)");
+        case NK::Cast: return ex(n->kids[0], pr);
+        case NK::LAnd: {
+            std::string a = def("(u32)(" + ex(n->kids[0], pr) + " != 0u)");
+            std::string p = def("(" + pr + ") & " + a);
+            std::string b = ex(n->kids[1], p);
+            return def(a + " & (u32)(" + b + " != 0u)");
+        }
+        case NK::LOr: {
+            std::string a = def("(u32)(" + ex(n->kids[0], pr) + " != 0u)");
+            std::string p = def("(" + pr + ") & (" + a + " ^ 1u)");
+            std::string b = ex(n->kids[1], p);
+            return def(a + " | (u32)(" + b + " != 0u)");
+        }
+        case NK::Select: {
+            std::string c = def("(u32)(" + ex(n->kids[0], pr) + " != 0u)");
+            std::string p1 = def("(" + pr + ") & " + c);
+            std::string p0 = def("(" + pr + ") & (" + c + " ^ 1u)");
+            std::string x = ex(n->kids[1], p1);
+            std::string y = ex(n->kids[2], p0);
+            return def(c + " ? " + x + " : " + y);
+        }
+        case NK::Min:
+        case NK::Max: {
+            std::string a = ex(n->kids[0], pr), b = ex(n->kids[1], pr);
+            std::string lt = n->opty == Ty::U32 ? "(" + a + " < " + b + ")" : "pg_slt(" + a + ", " + b + ")";
+            return def(n->kind == NK::Min ? lt + " ? " + a + " : " + b : lt + " ? " + b + " : " + a);
+        }
+        case NK::Bin: {
+            std::string a = ex(n->kids[0], pr), b = ex(n->kids[1], pr);
+            bool u = n->opty == Ty::U32;
+            switch (n->op) {
+            case Bop::Add: return def("pg_add(" + a + ", " + b + ")");
+            case Bop::Sub: return def("pg_sub(" + a + ", " + b + ")");
+            case Bop::Mul: return def("pg_mul(" + a + ", " + b + ")");
+            case Bop::Div: return def(std::string(u ? "pg_udiv(" : "pg_sdiv(") + a + ", " + b + ")");
+            case Bop::Rem: return def(std::string(u ? "pg_urem(" : "pg_srem(") + a + ", " + b + ")");
+            case Bop::Shl: return def("pg_shl(" + a + ", " + b + ")");
+            case Bop::Shr: return def(std::string(u ? "pg_lshr(" : "pg_ashr(") + a + ", " + b + ")");
+            case Bop::And: return def("(" + a + " & " + b + ")");
+            case Bop::Or: return def("(" + a + " | " + b + ")");
+            case Bop::Xor: return def("(" + a + " ^ " + b + ")");
+            case Bop::Lt: return def(u ? "(u32)(" + a + " < " + b + ")" : "pg_slt(" + a + ", " + b + ")");
+            case Bop::Le: return def(u ? "(u32)(" + a + " <= " + b + ")" : "pg_sle(" + a + ", " + b + ")");
+            case Bop::Gt: return def(u ? "(u32)(" + a + " > " + b + ")" : "pg_slt(" + b + ", " + a + ")");
+            case Bop::Ge: return def(u ? "(u32)(" + a + " >= " + b + ")" : "pg_sle(" + b + ", " + a + ")");
+            case Bop::Eq: return def("(u32)(" + a + " == " + b + ")");
+            case Bop::Ne: return def("(u32)(" + a + " != " + b + ")");
+            }
+        }
+        }
+        return "0u";
+    }
+    std::string def(const std::string& e) {
+        std::string r = tmp();
+        line("const u32 " + r + " = " + e + ";");
+        return r;
+    }
+
+    // ---------------------------------------------------------------- statements
+    void kill_preds(const std::string& k, size_t down_to) {
+        for (size_t i = preds.size(); i-- > down_to;) line(preds[i] + " &= " + k + " ^ 1u;");
+    }
+    void stmt(const Stmt* s) {
+        switch (s->kind) {
+        case SK::Seq:
+            for (const Stmt* c : s->seq) stmt(c);
+            return;
+        case SK::Nop: return;
+        case SK::Assign: {
+            line("{");
+            std::string v = ex(s->value, eff());
+            std::string dst = "F.v" + std::to_string(s->var);
+            if (uniform_ctx()) line(dst + " = " + v + ";");
+            else line(dst + " = " + eff() + " ? " + v + " : " + dst + ";");
+            line("}");
+            return;
+        }
+        case SK::Store: {
+            line("{");
+            const ArrayDecl& a = K.arrays[(size_t)s->arr];
+            Node tmpn;
+            tmpn.kids = s->index;
+            std::string pe = eff();
+            std::string f = flat_index(&tmpn, s->arr, pe);
+            std::string v = ex(s->value, pe);
+            std::string A = std::to_string(s->arr), S = std::to_string(s->site) + "u";
+            if (a.space == SHARED) line("pg_st_sh<" + A + ">(C, t, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
+            else if (a.space == GLOBAL) line("pg_st_gt<" + A + ">(C, t, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
+            else
+                line("if (pg_priv_ok(C, t, " + pe + ", " + f + ", " + hex(priv_size(a)) + ", " +
+                     hex(0x200u + (uint32_t)a.slot) + ", " + S + ", " + v + ", 1u)) F.p" + std::to_string(a.slot) +
+                     "[" + f + "] = " + v + ";");
+            line("}");
+            return;
+        }
+        case SK::PrivDecl: {
+            const ArrayDecl& a = K.arrays[(size_t)s->arr];
+            std::string pe = eff();
+            line("if (" + pe + ") { for (u32 _i = 0; _i < " + hex(priv_size(a)) + "; _i++) F.p" +
+                 std::to_string(a.slot) + "[_i] = 0u; }");
+            return;
+        }
+        case SK::If:
+            if (s->uniform) uniform_if(s);
+            else predicated_if(s);
+            return;
+        case SK::Loop:
+            if (s->uniform) uniform_loop(s);
+            else predicated_loop(s);
+            return;
+        case SK::Sync: {
+            int k = ++nsync;
+            line("return " + std::to_string(k) + "u;");
+            body << "R" << k << ":;\n";
+            return;
+        }
+        case SK::Return:
+            if (uniform_ctx()) {
+                line("t.live = 0u; return PG_END;");
+            } else {
+                line("{");
+                line("const u32 _k = " + eff() + ";");
+                line("t.live &= _k ^ 1u;");
+                kill_preds("_k", 0);
+                line("}");
+            }
+            return;
+        case SK::Break:
+        case SK::Continue: {
+            const Loop& L = loops.back();
+            if (L.uniform) {
+                line("goto L" + std::to_string(s->kind == SK::Break ? L.exit_label : L.cont_label) + ";");
+                return;
+            }
+            line("{");
+            line("const u32 _k = " + eff() + ";");
+            if (s->kind == SK::Break) line(L.act + " &= _k ^ 1u;");
+            kill_preds("_k", L.body_depth);
+            line("}");
+            return;
+        }
+        }
+    }
+    void uniform_if(const Stmt* s) {
+        int le = label(), lend = label();
+        line("{");
+        std::string c = ex(s->cond, "t.live");
+        line("if (!" + c + ") goto L" + std::to_string(le) + ";");
+        line("}");
+        stmt(s->body);
+        if (s->other) line("goto L" + std::to_string(lend) + ";");
+        body << "L" << le << ":;\n";
+        if (s->other) {
+            stmt(s->other);
+            body << "L" << lend << ":;\n";
+        }
+    }
+    void predicated_if(const Stmt* s) {
+        line("{");
+        std::string c = ex(s->cond, eff());
+        std::string pt = tmp("p"), pf = tmp("p");
+        line("u32 " + pt + " = " + cur() + " & (u32)(" + c + " != 0u);");
+        line("u32 " + pf + " = " + cur() + " & (u32)(" + c + " == 0u);");
+        line("if (__any_sync(PG_FULL, " + pt + " & t.live)) {");
+        preds.push_back(pt);
+        stmt(s->body);
+        preds.pop_back();
+        line("}");
+        if (s->other) {
+            line("if (__any_sync(PG_FULL, " + pf + " & t.live)) {");
+            preds.push_back(pf);
+            stmt(s->other);
+            preds.pop_back();
+            line("}");
+        }
+        line("}");
+    }
+    void uniform_loop(const Stmt* s) {
+        if (s->init) stmt(s->init);
+        Loop L;
+        L.id = s->loop;
+        L.uniform = true;
+        int head = label();
+        L.cont_label = label();
+        L.exit_label = label();
+        body << "L" << head << ":;\n";
+        if (s->cond) {
+            line("{");
+            std::string c = ex(s->cond, "t.live");
+            line("if (!" + c + ") goto L" + std::to_string(L.exit_label) + ";");
+            line("}");
+        }
+        loops.push_back(L);
+        stmt(s->body);
+        body << "L" << L.cont_label << ":;\n";
+        if (s->step) stmt(s->step);
+        loops.pop_back();
+        line("pg_tick(C, t, t.live);");
+        line("if (++C.ufuel > C.fuel) { t.live = 0u; return PG_END; }");
+        line("goto L" + std::to_string(head) + ";");
+        body << "L" << L.exit_label << ":;\n";
+    }
+    void predicated_loop(const Stmt* s) {
+        if (s->init) stmt(s->init);
+        line("{");
+        Loop L;
+        L.id = s->loop;
+        L.uniform = false;
+        L.act = tmp("a");
+        line("u32 " + L.act + " = " + cur() + ";");
+        line("for (;;) {");
+        if (s->cond) {
+            line("{");
+            std::string c = ex(s->cond, "(" + L.act + " & t.live)");
+            line(L.act + " &= (u32)(" + c + " != 0u);");
+            line("}");
+        }
+        line(L.act + " &= t.live;");
+        line("if (!__any_sync(PG_FULL, " + L.act + ")) break;");
+        std::string b = tmp("b");
+        line("{");
+        line("u32 " + b + " = " + L.act + ";");
+        preds.push_back(b);
+        L.body_depth = preds.size() - 1;
+        loops.push_back(L);
+        stmt(s->body);
+        loops.pop_back();
+        preds.pop_back();
+        line("}");
+        if (s->step) {
+            preds.push_back(L.act);
+            stmt(s->step);
+            preds.pop_back();
+        }
+        line("pg_tick(C, t, " + L.act + " & t.live);");
+        line("}");
+        line("}");
+    }
+
+    std::string run() {
+        stmt(K.body);
+        line("t.live = 0u; return PG_END;");
+        std::ostringstream o;
+        o << "#define PG_BITS " << O.bits << "\n";
+        o << "#define PG_RACECHK " << ((O.checks & 2) ? 1 : 0) << "\n";
+        o << "#define PG_OOBCHK " << ((O.checks & 4) ? 1 : 0) << "\n";
+        o << "#define PG_BANKCHK " << ((O.checks & 8) ? 1 : 0) << "\n";
+        o << "#define PG_COALCHK " << ((O.checks & 16) ? 1 : 0) << "\n";
+        o << "#define PG_BANK16 " << (O.bank_model == 1 ? 1 : 0) << "\n";
+        o << "#define PG_WMAX " << O.wmax << "\n";
+        o << "#define PG_NSTATS " << std::max<size_t>(1, K.sites.size()) << "\n";
+        o << "#ifndef PG_VMAX\n#define PG_VMAX 1\n#endif\n";
+        o << "#include \"pg_device_rt.cuh\"\n\n";
+        o << "// kernel " << K.name << "\n";
+        o << "struct PgK {\n  struct Frame {\n";
+        for (size_t i = 0; i < K.vars.size(); i++)
+            o << "    u32 v" << i << ";  // " << K.vars[i].name << (K.vars[i].uniform ? " (uniform)" : "") << "\n";
+        for (const ArrayDecl& a : K.arrays)
+            if (a.space == PRIVATE) o << "    u32 p" << a.slot << "[" << priv_size(a) << "];  // " << a.name << "\n";
+        o << "    u32 pad_;\n  };\n";
+        o << "  static __device__ __forceinline__ void init(Frame& F, const PgC& C, PgT& t) {\n";
+        for (size_t i = 0; i < K.vars.size(); i++) {
+            if (K.vars[i].scalar)
+                o << "    F.v" << i << " = pg_m((u32)C.L->scal[" << K.vars[i].scalar_index << "]);\n";
+            else
+                o << "    F.v" << i << " = 0u;\n";
+        }
+        o << "  }\n";
+        o << "  static __device__ __forceinline__ u32 seg(Frame& F, PgC& C, PgT& t, u64* ss, u32 resume) {\n";
+        o << "    switch (resume) {\n      case 0u: goto R0;\n";
+        for (int k = 1; k <= nsync; k++) o << "      case " << k << "u: goto R" << k << ";\n";
+        o << "      default: return PG_END;\n    }\n";
+        o << "R0:;\n" << body.str();
+        o << "  }\n};\n\n";
+        o << "extern \"C\" __global__ void __launch_bounds__(1024, 1) pgk_eval(const PgParams P) { pg_main<PgK>(P); }\n";
+        return o.str();
+    }
+};
+
+}  // namespace
+
+std::string generate_cuda(const Kernel& k, const CodegenOptions& opt) {
+    Gen g(k, opt);
+    return g.run();
+}
+
+}  // namespace pgf

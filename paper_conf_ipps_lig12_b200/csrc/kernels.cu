@@ -1,0 +1,261 @@
+// kernels.cu — ahead-of-time CUDA kernels of libpgvc (sm_100a):
+//   K1 pg_gen_inputs  : initial global-array contents from the PRF (H2, X7/X8)
+//   K3 pg_compare     : comparative assertion o_s = o_t (H7)
+//   K4 pg_summarize / pg_scan / pg_compact : canonical record list + counters (H8, X16)
+// The evaluation kernel K2 is generated per IR (codegen.cpp) and JIT-compiled.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "pg_layout.h"
+#include "pg_prf.cuh"
+
+namespace {
+
+__device__ __forceinline__ u32 init_value(u32 mode, u32 range, u32 mask, u64 seed, u32 gid, u32 i) {
+    u32 v;
+    if (mode == 1) v = i < 64 ? (u32)((seed >> i) & 1ull) : 0u;                 // BITS01
+    else if (mode == 2) v = pg_rand32(seed, gid, i) % (range ? range : 1u);      // RANGE(k)
+    else v = pg_rand32(seed, gid, i);                                           // RAND32
+    return v & mask;
+}
+
+// K1: blockIdx.y = job, blockIdx.x strides over the job's instances, threads
+// stride over the words.
+__global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ jobs, u32* arena_s, u32* arena_t,
+                                                     u32* input, u64 seed_base, u32 mode, u32 range, u32 mask) {
+    const PgFill f = jobs[blockIdx.y];
+    u32* region = f.target == 0 ? arena_s : f.target == 1 ? arena_t : input;
+    for (u32 inst = blockIdx.x; inst < f.n_inst; inst += gridDim.x) {
+        u32* base = region + f.dst + (u64)inst * f.stride;
+        const u64 seed = seed_base + (u64)f.j0 + (u64)inst * f.jstep;
+        if (f.op == PGF_CONST) {
+            for (u32 i = threadIdx.x; i < f.n; i += blockDim.x) base[i] = f.value;
+        } else if (f.op == PGF_INPUT) {
+            for (u32 i = threadIdx.x; i < f.n; i += blockDim.x) base[i] = init_value(mode, range, mask, seed, f.gid, i);
+        } else {
+            u64* cells = (u64*)base;
+            for (u32 i = threadIdx.x; i < f.n; i += blockDim.x)
+                cells[i] = ((u64)PG_NEVER << 32) | init_value(mode, range, mask, seed, f.gid, i);
+        }
+    }
+}
+
+__device__ __forceinline__ u32 cmp_val(const u32* region, u32 kind, u64 off, u32 i) {
+    return kind == 0 ? (u32)((const u64*)(region + off))[i] : region[off + i];
+}
+
+// K3a: count mismatching cells per (instance, array); keep the minimum (gid, addr)
+// per instance.
+__global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs, const u32* arena_s,
+                                                  const u32* arena_t, const u32* input, PgSlot* slots,
+                                                  u64* mm_key) {
+    __shared__ u32 s_cnt;
+    __shared__ u32 s_min;
+    const PgCmp c = jobs[blockIdx.y];
+    const u32* rs = c.src_kind == 0 ? arena_s : input;
+    const u32* rt = c.tgt_kind == 0 ? arena_t : input;
+    for (u32 inst = blockIdx.x; inst < c.n_inst; inst += gridDim.x) {
+        if (threadIdx.x == 0) { s_cnt = 0; s_min = PG_NEVER; }
+        __syncthreads();
+        const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
+        u32 cnt = 0, mn = PG_NEVER;
+        for (u32 i = threadIdx.x; i < c.n; i += blockDim.x) {
+            if (cmp_val(rs, c.src_kind, so, i) != cmp_val(rt, c.tgt_kind, to, i)) { cnt++; mn = min(mn, i); }
+        }
+        cnt = __reduce_add_sync(0xffffffffu, cnt);
+        mn = __reduce_min_sync(0xffffffffu, mn);
+        if ((threadIdx.x & 31) == 0 && cnt) { atomicAdd(&s_cnt, cnt); atomicMin(&s_min, mn); }
+        __syncthreads();
+        if (threadIdx.x == 0 && s_cnt) {
+            atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step].count, (u64)s_cnt);
+            atomicMin(&mm_key[c.inst0 + inst], ((u64)c.gid << 32) | s_min);
+        }
+        __syncthreads();
+    }
+}
+
+// K3b: fill the MISMATCH record of every failing instance from its minimum cell.
+__global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__ jobs, const u32* arena_s,
+                                                       const u32* arena_t, const u32* input, PgSlot* slots,
+                                                       const u64* mm_key) {
+    const PgCmp c = jobs[blockIdx.y];
+    const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
+    if (inst >= c.n_inst) return;
+    const u64 k = mm_key[c.inst0 + inst];
+    if (k == ~0ull || (u32)(k >> 32) != c.gid) return;
+    const u32 addr = (u32)k;
+    const u32* rs = c.src_kind == 0 ? arena_s : input;
+    const u32* rt = c.tgt_kind == 0 ? arena_t : input;
+    const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
+    PgSlot* s = &slots[c.slot0 + (u64)inst * c.slot_step];
+    s->f[0] = 0xFFFFu;
+    s->f[1] = c.gid;
+    s->f[2] = addr;
+    s->f[3] = c.src_kind == 0 ? arena_s[c.src_lw + (u64)inst * c.src_stride + addr] - 1u : PG_NEVER;
+    s->f[4] = c.tgt_kind == 0 ? arena_t[c.tgt_lw + (u64)inst * c.tgt_stride + addr] - 1u : PG_NEVER;
+    s->f[5] = PG_NEVER;
+    s->f[6] = cmp_val(rs, c.src_kind, so, addr);
+    s->f[7] = cmp_val(rt, c.tgt_kind, to, addr);
+    s->has = 1u;
+}
+
+__global__ void pg_reset_counters(long long* first_key, long long* counts) {
+    const u32 i = threadIdx.x;
+    if (i < 11) first_key[i] = 0x7FFFFFFFFFFFFFFFll;
+    if (i < 16) counts[i] = 0;
+}
+
+__device__ __forceinline__ bool kind_failing(u32 kind, u32 banks_mode) {
+    return kind <= PGK_MISMATCH || kind == PGK_LIMIT || (banks_mode && (kind == PGK_BANK || kind == PGK_UNCOAL));
+}
+
+// K4a: per instance (launch, local seed m): count non-empty slots, fold counts
+// and keys into the summary (X16/X17).
+__global__ void __launch_bounds__(256) pg_summarize(const PgSlot* __restrict__ slots, u32 n_inst, u32 n_local,
+                                                    u32 rank, u32 world, u32 banks_mode, u32* inst_nrec,
+                                                    long long* first_key, long long* counts) {
+    const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
+    if (inst >= n_inst) return;
+    const u32 li = inst / n_local, m = inst % n_local;
+    const u32 sj = rank + m * world;
+    u32 n = 0, failing = 0;
+    for (u32 k = 0; k < 2; k++) {
+        for (u32 kind = 0; kind < PG_NK; kind++) {
+            const PgSlot& s = slots[((u64)inst * 2 + k) * PG_NK + kind];
+            if (s.count == 0 || !s.has) continue;
+            n++;
+            const long long key = (long long)(((u64)li << 45) | ((u64)sj << 21) | ((u64)k << 20) |
+                                              ((u64)kind << 16) | (u64)(s.f[0] & 0xFFFFu));
+            atomicAdd((unsigned long long*)&counts[1 + kind], (unsigned long long)s.count);
+            atomicMin(&first_key[1 + kind], key);
+            if (kind_failing(kind, banks_mode)) {
+                failing = 1;
+                atomicMin(&first_key[0], key);
+            }
+        }
+    }
+    inst_nrec[inst] = n;
+    if (n) atomicAdd((unsigned long long*)&counts[11], (unsigned long long)n);
+    if (failing) atomicAdd((unsigned long long*)&counts[12], 1ull);
+}
+
+// K4b: exclusive scan of per-instance record counts (one CTA; chunked).
+__global__ void __launch_bounds__(1024) pg_scan(const u32* in, u64* out, u32 n) {
+    __shared__ u64 warp_sums[32];
+    __shared__ u64 carry;
+    if (threadIdx.x == 0) carry = 0;
+    __syncthreads();
+    for (u32 base = 0; base < n; base += 1024) {
+        const u32 i = base + threadIdx.x;
+        u64 v = i < n ? in[i] : 0;
+        const u32 lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+        u64 x = v;
+        for (int o = 1; o < 32; o <<= 1) {
+            u64 y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= (u32)o) x += y;
+        }
+        if (lane == 31) warp_sums[w] = x;
+        __syncthreads();
+        if (w == 0) {
+            u64 s = warp_sums[lane];
+            for (int o = 1; o < 32; o <<= 1) {
+                u64 y = __shfl_up_sync(0xffffffffu, s, o);
+                if (lane >= (u32)o) s += y;
+            }
+            warp_sums[lane] = s;
+        }
+        __syncthreads();
+        const u64 incl = x + (w ? warp_sums[w - 1] : 0) + carry;
+        if (i < n) out[i] = incl - v;
+        __syncthreads();
+        if (threadIdx.x == 1023) carry = incl;
+        __syncthreads();
+    }
+}
+
+struct PgCexDev {
+    u64 key, count;
+    u32 kind, launch, seed_idx, kernel, round, site, array, addr, tid_a, tid_b, val_a, val_b;
+};
+
+// K4c: write each instance's records at its scanned offset (slot order = key order).
+__global__ void __launch_bounds__(256) pg_compact(const PgSlot* __restrict__ slots, u32 n_inst, u32 n_local,
+                                                  u32 rank, u32 world, const u64* offsets, PgCexDev* out,
+                                                  u64 cap) {
+    const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
+    if (inst >= n_inst) return;
+    const u32 li = inst / n_local, m = inst % n_local;
+    const u32 sj = rank + m * world;
+    u64 o = offsets[inst];
+    for (u32 k = 0; k < 2; k++) {
+        for (u32 kind = 0; kind < PG_NK; kind++) {
+            const PgSlot& s = slots[((u64)inst * 2 + k) * PG_NK + kind];
+            if (s.count == 0 || !s.has) continue;
+            if (o < cap) {
+                PgCexDev r;
+                r.key = ((u64)li << 45) | ((u64)sj << 21) | ((u64)k << 20) | ((u64)kind << 16) | (u64)(s.f[0] & 0xFFFFu);
+                r.count = s.count;
+                r.kind = kind;
+                r.launch = li;
+                r.seed_idx = sj;
+                r.kernel = k;
+                r.round = s.f[0];
+                r.array = s.f[1];
+                r.addr = s.f[2];
+                r.tid_a = s.f[3];
+                r.tid_b = s.f[4];
+                r.site = s.f[5];
+                r.val_a = s.f[6];
+                r.val_b = s.f[7];
+                out[o] = r;
+            }
+            o++;
+        }
+    }
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ host wrappers (C++ linkage, used by api.cpp)
+namespace pgk {
+
+cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 max_inst, u32* arena_s, u32* arena_t, u32* input,
+                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st) {
+    for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
+        const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
+        dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
+        pg_gen_inputs<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, seed_base, mode, range, mask);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 max_inst, const u32* arena_s, const u32* arena_t,
+                    const u32* input, PgSlot* slots, u64* mm_key, cudaStream_t st) {
+    for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
+        const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
+        dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
+        pg_compare<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, slots, mm_key);
+        dim3 g2((max_inst + 127) / 128, nj);
+        pg_compare_fill<<<g2, 128, 0, st>>>(jobs + j0, arena_s, arena_t, input, slots, mm_key);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t reset_counters(long long* first_key, long long* counts, cudaStream_t st) {
+    pg_reset_counters<<<1, 32, 0, st>>>(first_key, counts);
+    return cudaGetLastError();
+}
+
+cudaError_t summarize_compact(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, u32 banks_mode,
+                              u32* inst_nrec, u64* offsets, void* out, u64 cap, long long* first_key,
+                              long long* counts, cudaStream_t st) {
+    if (!n_inst) return cudaSuccess;
+    pg_summarize<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, banks_mode, inst_nrec,
+                                                       first_key, counts);
+    pg_scan<<<1, 1024, 0, st>>>(inst_nrec, offsets, n_inst);
+    pg_compact<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, offsets,
+                                                     (PgCexDev*)out, cap);
+    return cudaGetLastError();
+}
+
+}  // namespace pgk

@@ -1,0 +1,108 @@
+// pg_layout.h — data layout shared by the host planner (api.cpp) and the
+// device runtime (device_rt.cuh, compiled by NVRTC).  Plain C structs only.
+#pragma once
+#ifndef __CUDACC_RTC__
+#include <stdint.h>
+#endif
+
+typedef unsigned int u32;
+typedef unsigned long long u64;
+typedef int i32;
+typedef unsigned short u16;
+
+#define PG_FULL 0xffffffffu
+#define PG_END 0xFFFFu
+#define PG_NEVER 0xFFFFFFFFu
+#define PG_NK 10
+#define PG_MAXARR 16
+
+enum { PGK_BARRIER_DIV = 0, PGK_OOB = 1, PGK_WW = 2, PGK_RW = 3, PGK_XB = 4, PGK_MISMATCH = 5, PGK_BANK = 6,
+       PGK_UNCOAL = 7, PGK_UNINIT = 8, PGK_LIMIT = 9 };
+enum { PGA_GT = 0, PGA_GI = 1, PGA_SH = 2, PGA_PR = 3 };
+
+// ------------------------------------------------------------------ shared host/device layout
+struct PgArr {
+    u32 size;       // flat words
+    u32 d1, d2;     // trailing dims for the row-major flat index
+    u32 kind;       // PGA_*
+    u32 rec_id;     // array id in records: gid | 0x100 + slot | 0x200 + slot
+    u32 gid;        // pair-level global id (PRF tag, X8)
+    u32 smem_cells; // shared: byte offset of u64 cells in the group region
+    u32 smem_wmax;  // shared: byte offset of u32 wmax stamps
+    u32 smem_rmin, smem_rmax;
+    u32 flags;      // bit0: reader stamps present (array read and written, race checks on)
+    u32 pad;
+    u64 off_cells;  // global tracked: u32-word offset of u64 cells in the instance arena
+    u64 off_lw;     // last committing writer (gtid + 1)
+    u64 off_wmax, off_rmin, off_rmax, off_xf, off_xl;
+    u64 off_in;     // global input: u32-word offset in the instance input region
+};
+
+struct PgLaunchK {
+    u32 gdim[3], bdim[3];
+    i32 scal[8];
+    u32 T, nblocks;
+    u32 lpg, gpw, wpg, V, P, cta_threads;
+    u32 smem_group_bytes, smem_cells_bytes;  // per group: cells region first, then u32 stamps
+    u32 n_arrays, smem_never_off;             // stamps in [cells_bytes, never_off) start at 0, the rest at ~0
+    u64 arena_stride, input_stride;          // u32 words per instance
+    PgArr arr[PG_MAXARR];
+};
+
+struct PgWork {
+    u32 launch;      // index into the launch table (and the record key)
+    u32 ngroups;     // instances in this CTA
+    u32 seed_j0;     // seed index of group 0
+    u32 seed_jstep;  // seed index stride between groups (= world)
+    u64 arena_off;   // u32-word offset of group 0's kernel arena
+    u64 input_off;   // u32-word offset of group 0's input region
+    u64 slot0;       // slot index (instance, this kernel, kind 0) of group 0
+    u64 slot_step;   // slot stride between groups
+};
+
+struct PgSlot {
+    u64 count;
+    u32 lock, has;
+    u32 f[8];  // round, array, addr, tid_a, tid_b, site, val_a, val_b
+};
+
+struct PgParams {
+    const PgLaunchK* launches;
+    const PgWork* work;
+    u32* arena;
+    const u32* input;
+    PgSlot* slots;
+    u64* counts;       // d_counts (int64[16] viewed as u64)
+    u64* site_stats;   // [n_launch][max_sites][8] for this kernel, or null
+    u64 seed_base;
+    u32 max_sites;
+    u32 kernel_idx;
+    u32 fuel;
+    u32 pad;
+};
+
+
+// K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive
+// instances of one launch (instance i at dst + i * stride, seed index j0 + i * jstep).
+enum { PGF_CONST = 0, PGF_CELLS = 1, PGF_INPUT = 2 };
+struct PgFill {
+    u64 dst;      // u32-word offset of instance 0 in the target region
+    u64 stride;   // u32 words between instances
+    u32 n;        // elements (u32 for CONST/INPUT, u64 cells for CELLS)
+    u32 n_inst;
+    u32 j0, jstep;
+    u32 op;       // PGF_*
+    u32 gid;      // PRF tag (X8)
+    u32 value;    // PGF_CONST fill value
+    u32 target;   // 0 arena (src), 1 arena (tgt), 2 input region
+};
+
+// K3 (pg_compare) job: one compared global array for n_inst consecutive
+// instances of one launch (H7).
+struct PgCmp {
+    u64 src_off, tgt_off;        // u32-word offsets of instance 0: u64 cells in an arena (kind 0) or u32 input (kind 1)
+    u64 src_stride, tgt_stride;  // per-instance strides of the regions the offsets point into
+    u64 src_lw, tgt_lw;          // last-writer words of instance 0 (kind 0 only)
+    u64 slot0, slot_step;        // MISMATCH slot of (instance 0, kernel 0) and stride
+    u32 inst0, n_inst, gid, n, src_kind, tgt_kind;
+};

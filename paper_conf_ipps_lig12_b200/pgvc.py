@@ -1,0 +1,260 @@
+"""ctypes binding of libpgvc.so (include/pgvc.h) — argument marshalling only.
+
+Every step of the checked path runs in the library's CUDA kernels; this module
+only converts Python launch lists and torch tensors into the C structs.  It
+loads the in-tree libpgvc.so and raises if it is missing: there is no CPU
+fallback (use `python -m paper_conf_ipps_lig12_b200.build` to compile it).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+from typing import List, Optional, Sequence
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libpgvc.so")
+
+PG_OK, PG_E_ARG, PG_E_PARSE, PG_E_TYPE, PG_E_LIMIT, PG_E_CUDA, PG_E_OOM, PG_E_STATE = 0, -1, -2, -3, -4, -5, -6, -7
+IN_RAND32, IN_BITS01, IN_RANGE = 0, 1, 2
+CHK_EQUIV, CHK_RACE, CHK_OOB, CHK_BANK, CHK_COALESCE = 1, 2, 4, 8, 16
+BANKS_32, BANKS_16_HALFWARP = 0, 1
+KINDS = ["BARRIER_DIV", "OOB", "RACE_WW", "RACE_RW", "RACE_XB", "MISMATCH", "BANK", "UNCOALESCED", "UNINIT", "LIMIT"]
+N_KINDS = 10
+FAILING = {0, 1, 2, 3, 4, 5, 9}
+
+
+class PgLaunch(ctypes.Structure):
+    _fields_ = [("gdim", ctypes.c_uint32 * 3), ("bdim", ctypes.c_uint32 * 3), ("scalar", ctypes.c_int32 * 8),
+                ("n_scalar", ctypes.c_uint32)]
+
+
+class PgSpace(ctypes.Structure):
+    _fields_ = [("launch_src", ctypes.POINTER(PgLaunch)), ("launch_tgt", ctypes.POINTER(PgLaunch)),
+                ("n_launch", ctypes.c_uint32), ("seed_base", ctypes.c_uint64), ("n_seeds", ctypes.c_uint32),
+                ("input_mode", ctypes.c_uint32), ("input_range", ctypes.c_uint32), ("bits", ctypes.c_uint32),
+                ("checks", ctypes.c_uint32), ("bank_model", ctypes.c_uint32), ("max_cex", ctypes.c_uint32),
+                ("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("cuda_stream", ctypes.c_void_p),
+                ("d_first_key", ctypes.c_void_p), ("d_counts", ctypes.c_void_p)]
+
+
+REC_FIELDS = ("key", "count", "kind", "launch", "seed_idx", "kernel", "round", "site", "array", "addr",
+              "tid_a", "tid_b", "val_a", "val_b")
+
+
+class PgCex(ctypes.Structure):
+    _fields_ = [("key", ctypes.c_uint64), ("count", ctypes.c_uint64)] + [
+        (n, ctypes.c_uint32) for n in REC_FIELDS[2:]]
+
+
+class PgSummary(ctypes.Structure):
+    _fields_ = [("instances", ctypes.c_uint64), ("n_fail", ctypes.c_uint64), ("n_records", ctypes.c_uint64),
+                ("first_key", ctypes.c_int64), ("first_launch", ctypes.c_uint32),
+                ("first_seed_idx", ctypes.c_uint32), ("per_kind", ctypes.c_uint64 * N_KINDS),
+                ("first_key_kind", ctypes.c_int64 * N_KINDS)]
+
+
+class PgError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__("pgvc error %d: %s" % (code, msg))
+        self.code = code
+
+
+_lib = None
+EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_collect_cex",
+           "pg_collect_site_stats", "pg_ir_info", "pg_ir_source", "pg_ir_compile", "pg_run_timing",
+           "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
+
+
+def lib():
+    """Load the in-tree libpgvc.so (raises if it has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError("libpgvc.so not built (run __graft_entry__.build() or python -m "
+                          "paper_conf_ipps_lig12_b200.build); there is no CPU fallback")
+    L = ctypes.CDLL(LIB_PATH)
+    vp = ctypes.c_void_p
+    L.pg_load_ir.argtypes = [ctypes.c_char_p, ctypes.c_size_t, ctypes.POINTER(vp)]
+    L.pg_check_equiv.argtypes = [vp, vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
+    L.pg_check_races.argtypes = [vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
+    L.pg_check_banks.argtypes = [vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
+    L.pg_collect_cex.argtypes = [vp, ctypes.POINTER(PgCex), ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t),
+                                 ctypes.POINTER(PgSummary)]
+    L.pg_collect_site_stats.argtypes = [vp, ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32]
+    L.pg_ir_info.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32),
+                             ctypes.POINTER(ctypes.c_uint32)]
+    L.pg_ir_source.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_char_p,
+                               ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]
+    L.pg_ir_compile.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32]
+    L.pg_run_timing.argtypes = [vp, ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_float),
+                                ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint64)]
+    L.pg_last_error.restype = ctypes.c_char_p
+    L.pg_version.restype = ctypes.c_char_p
+    L.pg_ir_free.argtypes = [vp]
+    L.pg_run_free.argtypes = [vp]
+    for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_collect_cex",
+              "pg_collect_site_stats", "pg_ir_info", "pg_ir_source", "pg_ir_compile", "pg_run_timing"):
+        getattr(L, f).restype = ctypes.c_int
+    _lib = L
+    return L
+
+
+def _ck(rc: int):
+    if rc != PG_OK:
+        raise PgError(rc, lib().pg_last_error().decode())
+
+
+class Ir:
+    """A loaded kernel (pg_load_ir)."""
+
+    def __init__(self, text: str):
+        self.text = text
+        self._h = ctypes.c_void_p()
+        b = text.encode()
+        _ck(lib().pg_load_ir(b, len(b), ctypes.byref(self._h)))
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self):
+        s, g, c = ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint32()
+        _ck(lib().pg_ir_info(self._h, ctypes.byref(s), ctypes.byref(g), ctypes.byref(c)))
+        return {"sites": s.value, "globals": g.value, "scalars": c.value}
+
+    def source(self, bits=32, checks=CHK_RACE | CHK_OOB, bank_model=0) -> str:
+        n = ctypes.c_size_t()
+        _ck(lib().pg_ir_source(self._h, bits, checks, bank_model, None, 0, ctypes.byref(n)))
+        buf = ctypes.create_string_buffer(n.value + 1)
+        _ck(lib().pg_ir_source(self._h, bits, checks, bank_model, buf, n.value + 1, ctypes.byref(n)))
+        return buf.value.decode()
+
+    def compile(self, bits=32, checks=CHK_RACE | CHK_OOB, bank_model=0):
+        _ck(lib().pg_ir_compile(self._h, bits, checks, bank_model))
+
+    def __del__(self):
+        if getattr(self, "_h", None) and self._h.value and _lib is not None:
+            _lib.pg_ir_free(self._h)
+            self._h = ctypes.c_void_p()
+
+
+def load_ir(text: str) -> Ir:
+    return Ir(text)
+
+
+def _launch(l) -> PgLaunch:
+    gdim, bdim, sc = (l.gdim, l.bdim, l.scalars) if hasattr(l, "gdim") else l
+    o = PgLaunch()
+    for i in range(3):
+        o.gdim[i] = gdim[i]
+        o.bdim[i] = bdim[i]
+    for i, v in enumerate(sc):
+        o.scalar[i] = v
+    o.n_scalar = len(sc)
+    return o
+
+
+@dataclass
+class Space:
+    """Python side of pg_space.  Launches are Launch objects or (gdim, bdim, scalars)."""
+    launch_src: Sequence
+    launch_tgt: Optional[Sequence] = None
+    n_seeds: int = 1
+    seed_base: int = 0
+    input_mode: int = IN_RAND32
+    input_range: int = 0
+    bits: int = 32
+    checks: int = CHK_EQUIV | CHK_RACE | CHK_OOB
+    bank_model: int = BANKS_32
+    max_cex: int = 1 << 20
+    rank: int = 0
+    world: int = 1
+    stream: int = 0                 # cudaStream_t as an integer (torch.cuda.Stream.cuda_stream)
+    first_key: object = None        # torch int64[11] on the device (optional)
+    counts: object = None           # torch int64[16] on the device (optional)
+
+    def marshal(self):
+        ls = (PgLaunch * max(1, len(self.launch_src)))(*[_launch(l) for l in self.launch_src])
+        lt = None
+        if self.launch_tgt is not None:
+            lt = (PgLaunch * max(1, len(self.launch_tgt)))(*[_launch(l) for l in self.launch_tgt])
+        sp = PgSpace()
+        sp.launch_src = ctypes.cast(ls, ctypes.POINTER(PgLaunch))
+        sp.launch_tgt = ctypes.cast(lt, ctypes.POINTER(PgLaunch)) if lt is not None else None
+        sp.n_launch = len(self.launch_src)
+        sp.seed_base = self.seed_base
+        sp.n_seeds = self.n_seeds
+        sp.input_mode, sp.input_range, sp.bits = self.input_mode, self.input_range, self.bits
+        sp.checks, sp.bank_model, sp.max_cex = self.checks, self.bank_model, self.max_cex
+        sp.rank, sp.world = self.rank, self.world
+        sp.cuda_stream = self.stream or None
+        sp.d_first_key = self.first_key.data_ptr() if self.first_key is not None else None
+        sp.d_counts = self.counts.data_ptr() if self.counts is not None else None
+        return sp, (ls, lt)
+
+
+class Run:
+    """Result set of one check (pg_run).  collect() synchronises its stream."""
+
+    def __init__(self, h, space: Space, keep):
+        self._h = h
+        self.space = space
+        self._keep = keep
+
+    def collect(self, cap: int = 1 << 20):
+        n = ctypes.c_size_t()
+        summ = PgSummary()
+        buf = (PgCex * max(1, cap))()
+        _ck(lib().pg_collect_cex(self._h, buf, cap, ctypes.byref(n), ctypes.byref(summ)))
+        m = min(n.value, cap)
+        recs = [tuple(getattr(buf[i], f) for f in REC_FIELDS) for i in range(m)]
+        s = {"instances": summ.instances, "n_fail": summ.n_fail, "n_records": summ.n_records,
+             "first_key": summ.first_key, "first_launch": summ.first_launch,
+             "first_seed_idx": summ.first_seed_idx, "per_kind": list(summ.per_kind),
+             "first_key_kind": list(summ.first_key_kind)}
+        return recs, s
+
+    def site_stats(self, max_sites: int):
+        import numpy as np
+        nl = len(self.space.launch_src)
+        out = np.zeros((nl, 2, max_sites, 8), dtype=np.uint64)
+        _ck(lib().pg_collect_site_stats(self._h, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), max_sites))
+        return out
+
+    def timing(self):
+        a, b, n, h = ctypes.c_float(), ctypes.c_float(), ctypes.c_uint32(), ctypes.c_uint64()
+        _ck(lib().pg_run_timing(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(n), ctypes.byref(h)))
+        return {"ms_eval": a.value, "ms_total": b.value, "launches": n.value, "h2d_bytes": h.value}
+
+    def __del__(self):
+        if getattr(self, "_h", None) and self._h.value and _lib is not None:
+            _lib.pg_run_free(self._h)
+            self._h = ctypes.c_void_p()
+
+
+def _run(fn, irs, space: Space) -> Run:
+    sp, keep = space.marshal()
+    h = ctypes.c_void_p()
+    _ck(fn(*[i.handle for i in irs], ctypes.byref(sp), ctypes.byref(h)))
+    return Run(h, space, (keep, irs))
+
+
+def pg_check_equiv(src: Ir, tgt: Ir, space: Space) -> Run:
+    return _run(lib().pg_check_equiv, [src, tgt], space)
+
+
+def pg_check_races(k: Ir, space: Space) -> Run:
+    return _run(lib().pg_check_races, [k], space)
+
+
+def pg_check_banks(k: Ir, space: Space) -> Run:
+    return _run(lib().pg_check_banks, [k], space)
+
+
+check_equiv, check_races, check_banks = pg_check_equiv, pg_check_races, pg_check_banks
+
+
+def version() -> str:
+    return lib().pg_version().decode()
