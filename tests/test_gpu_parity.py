@@ -31,6 +31,10 @@ def run_pair(env, oracle, src, tgt, ls, lt=None, mode=0, max_sites=0, **kw):
     pgvc, torch = env
     lt = lt if lt is not None else (ls if tgt else None)
     okw = {k: v for k, v in kw.items() if k in KW_ORACLE}
+    if mode == 1:       # pg_check_races: checks = RACE | OOB
+        okw["checks"] = oracle.RACE | oracle.OOB
+    elif mode == 2:     # pg_check_banks: checks = BANK | COALESCE
+        okw["checks"] = oracle.BANK | oracle.COALESCE
     ref = oracle.check(src, tgt, ls, lt, mode=mode, max_sites=max_sites, cap=1 << 20, **okw)
     sp = pgvc.Space(ls, lt, stream=torch.cuda.current_stream().cuda_stream, **kw)
     if mode == 0:
