@@ -182,6 +182,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--ref-log-n", type=int, default=12)
     ap.add_argument("--ref-seeds", type=int, default=4)
+    ap.add_argument("--profile", action="store_true", help="1 warm-up + 1 step, no JSON (for ncu launch lists)")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)
@@ -239,9 +240,15 @@ def main():
         return d2h, recs_total
 
     # warm-up (also JIT-compiles every evaluation kernel variant)
-    for _ in range(max(3, args.warmup)):
+    for _ in range(1 if args.profile else max(3, args.warmup)):
         collect(step())
     torch.cuda.synchronize()
+    if args.profile:
+        torch.cuda.cudart().cudaProfilerStart()
+        collect(step())
+        torch.cuda.synchronize()
+        torch.cuda.cudart().cudaProfilerStop()
+        return
 
     clocks = Clocks(local)
     if world > 1:

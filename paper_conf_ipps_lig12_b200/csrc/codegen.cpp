@@ -89,7 +89,7 @@ struct Gen {
             int c = n->ref % 3;
             std::string src;
             if (n->ref < 3) src = "t.tid[" + std::to_string(c) + "]";
-            else if (n->ref < 6) src = "C.bid[" + std::to_string(c) + "]";
+            else if (n->ref < 6) src = "t.bid[" + std::to_string(c) + "]";
             else if (n->ref < 9) src = "C.L->bdim[" + std::to_string(c) + "]";
             else src = "C.L->gdim[" + std::to_string(c) + "]";
             return "pg_m(" + src + ")";

@@ -61,7 +61,6 @@ __device__ __forceinline__ u32 pg_not(u32 a) { return pg_m(~a); }
 // ------------------------------------------------------------------ state
 struct PgC {                 // CTA-uniform state
     const PgLaunchK* L;      // in shared memory
-    u32 blk, bid[3];
     u32 round;               // round index within the block (record field)
     u32 step;                // round index within the instance, 1-based (stamps)
     u32 fuel;
@@ -70,6 +69,7 @@ struct PgC {                 // CTA-uniform state
 
 struct PgT {                 // per emulated thread
     u32 live;                // 0/1: not exited and a real thread of a real instance
+    u32 blk, bid[3];         // emulated block (linear id and bid.xyz)
     u32 tid[3];
     u32 tlin, gtid;
     u32 lane, ekey;          // HW lane; emulated-warp key within the HW warp (63: idle lane)
@@ -199,7 +199,7 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, u64* ss, u32 pe, u32 fla
 #endif
     if (!pe) return 0u;
     if (!inb) {
-        u32 pv = pg_m(pg_rand32(t.seed, 0x8000u + (a.rec_id - 0x100u), ((u64)C.blk << 20) + flat));
+        u32 pv = pg_m(pg_rand32(t.seed, 0x8000u + (a.rec_id - 0x100u), ((u64)t.blk << 20) + flat));
 #if PG_OOBCHK
         pg_event(t, PGK_OOB, C.round, a.rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
 #endif
@@ -216,7 +216,7 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, u64* ss, u32 pe, u32 fla
         if (t.lcell[i] == cell) return t.lval[i];
     const u64 c = ((const u64*)(t.sgrp + a.smem_cells))[flat];
     if ((u32)(c >> 32) == PG_NEVER) {
-        u32 pv = pg_m(pg_rand32(t.seed, 0x8000u + (a.rec_id - 0x100u), ((u64)C.blk << 20) + flat));
+        u32 pv = pg_m(pg_rand32(t.seed, 0x8000u + (a.rec_id - 0x100u), ((u64)t.blk << 20) + flat));
 #if PG_OOBCHK
         pg_event(t, PGK_UNINIT, C.round, a.rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
 #endif
@@ -261,16 +261,15 @@ __device__ __forceinline__ void pg_st_sh(PgC& C, PgT& t, u64* ss, u32 pe, u32 fl
 }
 
 // Global array written by this kernel: u64 cells in the instance arena.
+// XB bookkeeping (X4): first and last block that accessed a global cell.  Kept
+// whenever the launch has more than one block (it also decides whether the
+// block-parallel pass must be redone sequentially).
 template <int A>
 __device__ __forceinline__ void pg_xb_mark(const PgC& C, PgT& t, const PgArr& a, u32 flat) {
-#if PG_RACECHK
-    if (C.L->nblocks > 1) {
-        u32* xf = t.arena + a.off_xf;
-        u32* xl = t.arena + a.off_xl;
-        if (xf[flat] == 0u) xf[flat] = C.blk + 1u;
-        xl[flat] = C.blk + 1u;
+    if (a.off_xf != ~0ull) {
+        atomicMin(t.arena + a.off_xf + flat, t.blk + 1u);
+        atomicMax(t.arena + a.off_xl + flat, t.blk + 1u);
     }
-#endif
 }
 
 template <int A, bool RD>
@@ -441,17 +440,31 @@ __device__ __noinline__ void pg_flush(const PgParams& P, PgT& t, u64 slot0) {
 }
 
 // ------------------------------------------------------------------ CTA main loop
-// One CTA = P instances (groups) of one launch, in lock step: every group runs
-// the same blocks in linear bid order and the same (uniform) round structure.
+// A CTA runs P groups of one launch in lock step.  Group g emulates, for seed
+// (g / gb) of the work item, the blocks blk0 + i*gb + (g % gb), i = 0, 1, ...
+// (gb > 1 only when no block-uniform branch depends on bid, so all groups share
+// one round structure).  Blocks of one instance therefore run in parallel
+// (across groups and CTAs); that is exact unless a global cell is shared
+// between blocks (XB), which K2b detects - those seed groups are re-run by the
+// sequential pass (P.seq = 1: gb = 1, all blocks in linear bid order, X21).
 #ifndef PG_VMAX
 #define PG_VMAX 1
 #endif
+
+__device__ __forceinline__ u32 pg_init_value(const PgParams& P, u64 seed, u32 gid, u32 i) {
+    u32 v;
+    if (P.input_mode == 1) v = i < 64 ? (u32)((seed >> i) & 1ull) : 0u;
+    else if (P.input_mode == 2) v = pg_rand32(seed, gid, i) % (P.input_range ? P.input_range : 1u);
+    else v = pg_rand32(seed, gid, i);
+    return v & P.mask;
+}
 
 template <class K>
 __device__ __forceinline__ void pg_main(const PgParams& P) {
     extern __shared__ __align__(16) unsigned char pg_dsmem[];
     __shared__ PgLaunchK sL;
     __shared__ PgWork sW;
+    __shared__ u32 s_flag;
     {
         const u32* src = (const u32*)&P.launches[P.work[blockIdx.x].launch];
         u32* dst = (u32*)&sL;
@@ -462,7 +475,43 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
     }
     __syncthreads();
     const PgLaunchK& L = sL;
-    const u32 G = sW.ngroups;
+    const u32 G = sW.ngroups, GB = sW.gb;
+    if (P.seq) {
+        // re-run only seed groups in which some instance shared a global cell between blocks
+        if (threadIdx.x == 0) {
+            u32 f = 0;
+            for (u32 i = 0; i < sW.nseeds; i++) f |= P.xb_flag[sW.inst0 + i];
+            s_flag = f;
+        }
+        __syncthreads();
+        if (!s_flag) return;
+        // fresh arenas and slots for every seed of the group (the parallel pass is discarded)
+        for (u32 ms = 0; ms < sW.nseeds; ms++) {
+            const u64 seed = P.seed_base + (u64)(sW.seed_j0 + ms * sW.seed_jstep);
+            u32* ar = P.arena + sW.arena_off + (u64)ms * L.arena_stride;
+            for (u32 a = 0; a < L.n_arrays; a++) {
+                const PgArr& R = L.arr[a];
+                if (R.kind != PGA_GT) continue;
+                u64* cells = (u64*)(ar + R.off_cells);
+                for (u32 i = threadIdx.x; i < R.size; i += blockDim.x) {
+                    cells[i] = ((u64)PG_NEVER << 32) | pg_init_value(P, seed, R.gid, i);
+                    ar[R.off_lw + i] = 0u;
+                    if (R.off_wmax != ~0ull) ar[R.off_wmax + i] = 0u;
+                    if (R.off_rmin != ~0ull) ar[R.off_rmin + i] = PG_NEVER;
+                    if (R.off_rmax != ~0ull) ar[R.off_rmax + i] = 0u;
+                    if (R.off_xf != ~0ull) { ar[R.off_xf + i] = PG_NEVER; ar[R.off_xl + i] = 0u; }
+                }
+            }
+            if (threadIdx.x < PG_NK) {
+                PgSlot* sl = P.slots + sW.slot0 + (u64)ms * sW.slot_step + threadIdx.x;
+                sl->count = 0;
+                sl->has = 0;
+                sl->lock = 0;
+            }
+        }
+        __threadfence();
+        __syncthreads();
+    }
     unsigned char* sgroups = pg_dsmem;
     u64* sstats = (u64*)(pg_dsmem + (u64)L.P * L.smem_group_bytes);
     u32* s_alive = (u32*)(sstats + ((PG_BANKCHK || PG_COALCHK) ? PG_NSTATS * 8 : 0));
@@ -496,6 +545,7 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
     }
     const u32 inst_ok = lane_ok && g < G;
     const u32 gc = inst_ok ? g : 0u;
+    const u32 ms = gc / GB, bs = gc % GB;
     typename K::Frame F[PG_VMAX];
     PgT T[PG_VMAX];
     const u32 V = PG_VMAX > 1 ? L.V : 1u;
@@ -510,18 +560,17 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         t.tid[0] = t.tlin % L.bdim[0];
         t.tid[1] = (t.tlin / L.bdim[0]) % L.bdim[1];
         t.tid[2] = t.tlin / (L.bdim[0] * L.bdim[1]);
-        t.seed = P.seed_base + (u64)(sW.seed_j0 + gc * sW.seed_jstep);
-        t.arena = P.arena + sW.arena_off + (u64)gc * L.arena_stride;
-        t.input = P.input + sW.input_off + (u64)gc * L.input_stride;
+        t.seed = P.seed_base + (u64)(sW.seed_j0 + ms * sW.seed_jstep);
+        t.arena = P.arena + sW.arena_off + (u64)ms * L.arena_stride;
+        t.input = P.input + sW.input_off + (u64)ms * L.input_stride;
         t.sgrp = sgroups + (u64)gc * L.smem_group_bytes;
         for (u32 k = 0; k < PG_NK; k++) t.ecnt[k] = 0;
         t.live = ok;
     }
-    for (u32 blk = 0; blk < L.nblocks; blk++) {
-        C.blk = blk;
-        C.bid[0] = blk % L.gdim[0];
-        C.bid[1] = (blk / L.gdim[0]) % L.gdim[1];
-        C.bid[2] = blk / (L.gdim[0] * L.gdim[1]);
+    const u32 nsteps = (sW.blk1 - sW.blk0 + GB - 1) / GB;
+    for (u32 st = 0; st < nsteps; st++) {
+        const u32 blk = sW.blk0 + st * GB + bs;
+        const u32 blk_ok = blk < sW.blk1;
         // fresh shared arrays for every group: cells never written, stamps cleared
         {
             const u32 cw = L.smem_cells_bytes / 8u;
@@ -537,14 +586,22 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
                 for (u32 i = threadIdx.x; i < nw; i += blockDim.x) nv[i] = PG_NEVER;
             }
         }
-        for (u32 i = threadIdx.x; i < L.P; i += blockDim.x) { s_alive[i] = i < G; s_rounds[i] = 0; }
+        for (u32 i = threadIdx.x; i < L.P; i += blockDim.x) {
+            s_alive[i] = i < G && sW.blk0 + st * GB + (i % GB) < sW.blk1;
+            s_rounds[i] = 0;
+        }
         __syncthreads();
 #pragma unroll
         for (u32 v = 0; v < PG_VMAX; v++) {
             if (v >= V) break;
-            T[v].live = inst_ok && T[v].tlin < L.T;
-            T[v].gtid = blk * L.T + T[v].tlin;
-            K::init(F[v], C, T[v]);
+            PgT& t = T[v];
+            t.blk = blk;
+            t.bid[0] = blk % L.gdim[0];
+            t.bid[1] = (blk / L.gdim[0]) % L.gdim[1];
+            t.bid[2] = blk / (L.gdim[0] * L.gdim[1]);
+            t.live = inst_ok && t.tlin < L.T && blk_ok;
+            t.gtid = blk * L.T + t.tlin;
+            K::init(F[v], C, t);
         }
         C.round = 0;
         u32 resume = 0;
@@ -589,8 +646,9 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         __syncthreads();
     }
 #if PG_RACECHK
-    // X4: cross-block races on global cells written by this kernel
-    if (L.nblocks > 1) {
+    // X4: cross-block races on global cells written by this kernel (sequential pass: the
+    // CTA owns whole instances; the parallel pass leaves them to the flagged re-run)
+    if (P.seq && L.nblocks > 1) {
 #pragma unroll
         for (u32 v = 0; v < PG_VMAX; v++) {
             if (v >= V) break;
@@ -598,7 +656,7 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
             if (!(inst_ok && t.tlin < L.T)) continue;
             for (u32 a = 0; a < L.n_arrays; a++) {
                 const PgArr& ar = L.arr[a];
-                if (ar.kind != PGA_GT) continue;
+                if (ar.kind != PGA_GT || ar.off_xf == ~0ull) continue;
                 const u32* xf = t.arena + ar.off_xf;
                 const u32* xl = t.arena + ar.off_xl;
                 const u32* lw = t.arena + ar.off_lw;
@@ -613,13 +671,13 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
 #pragma unroll
     for (u32 v = 0; v < PG_VMAX; v++) {
         if (v >= V) break;
-        if (inst_ok && T[v].tlin < L.T) pg_flush(P, T[v], sW.slot0 + (u64)g * sW.slot_step);
+        if (inst_ok && T[v].tlin < L.T) pg_flush(P, T[v], sW.slot0 + (u64)ms * sW.slot_step);
     }
-    if (inst_ok && tl0 == 0u) atomicAdd(&P.counts[0], s_inst[g]);
+    if (!P.seq && inst_ok && tl0 == 0u) atomicAdd(&P.counts[0], s_inst[g]);
 #if PG_BANKCHK || PG_COALCHK
     __syncthreads();
     if (P.site_stats) {
-        u64* dst = P.site_stats + (u64)sW.launch * P.max_sites * 8u;
+        u64* dst = P.site_stats + (u64)(P.seq ? sW.launch : sW.item) * P.max_sites * 8u;
         for (u32 i = threadIdx.x; i < PG_NSTATS * 8 && i < P.max_sites * 8; i += blockDim.x) {
             const u32 c = i & 7u;
             if (c == 3) atomicMax(&dst[i], sstats[i]);

@@ -836,12 +836,53 @@ public:
         } while (changed_);
         mark_nodes(K.body);
         check_syncs(K.body, true);
+        // grid uniformity: variables whose uniform value never depends on bid
+        grid_.assign(K.vars.size(), true);
+        for (size_t v = 0; v < K.vars.size(); v++) grid_[v] = K.vars[v].uniform;
+        do {
+            changed_ = false;
+            grid_walk(K.body);
+        } while (changed_);
+        K.grid_uniform_control = grid_control(K.body);
     }
 
 private:
     Kernel& K;
     std::vector<bool> loop_nonuniform_jump_;
+    std::vector<bool> grid_;
     bool changed_ = false;
+
+    bool grid_uniform(const Node* n) const {
+        switch (n->kind) {
+        case NK::Lit: return true;
+        case NK::Var: return grid_[(size_t)n->ref];
+        case NK::Builtin: return n->ref >= 6;  // bdim, gdim
+        case NK::Elem: return false;
+        default:
+            for (const Node* c : n->kids)
+                if (!grid_uniform(c)) return false;
+            return true;
+        }
+    }
+    void grid_walk(const Stmt* s) {
+        if (!s) return;
+        if (s->kind == SK::Assign && grid_[(size_t)s->var] && !grid_uniform(s->value)) {
+            grid_[(size_t)s->var] = false;
+            changed_ = true;
+        }
+        for (const Stmt* c : s->seq) grid_walk(c);
+        grid_walk(s->body);
+        grid_walk(s->other);
+        grid_walk(s->init);
+        grid_walk(s->step);
+    }
+    bool grid_control(const Stmt* s) const {
+        if (!s) return true;
+        if ((s->kind == SK::If || s->kind == SK::Loop) && s->uniform && s->cond && !grid_uniform(s->cond)) return false;
+        for (const Stmt* c : s->seq)
+            if (!grid_control(c)) return false;
+        return grid_control(s->body) && grid_control(s->other) && grid_control(s->init) && grid_control(s->step);
+    }
 
     bool uniform(const Node* n) const {
         switch (n->kind) {

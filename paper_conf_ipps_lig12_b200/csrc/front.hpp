@@ -96,6 +96,10 @@ struct Kernel {
     std::vector<SiteInfo> sites;
     int n_loops = 0;
     int n_syncs = 0;
+    // every block-uniform branch / loop condition is also grid-uniform (does not
+    // depend on bid): emulated blocks with different bid share one round structure
+    // and can run lock-step in one CTA
+    bool grid_uniform_control = true;
     Stmt* body = nullptr;
     std::vector<std::unique_ptr<Node>> node_pool;
     std::vector<std::unique_ptr<Stmt>> stmt_pool;

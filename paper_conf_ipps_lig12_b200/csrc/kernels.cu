@@ -99,6 +99,46 @@ __global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__
     s->has = 1u;
 }
 
+// K2b: flag every instance in which some global cell written by the kernel was
+// accessed by two blocks (X4 XB) - the block-parallel pass is not exact there.
+__global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ jobs, const u32* arena, u32* flags) {
+    const PgXb j = jobs[blockIdx.y];
+    for (u32 inst = blockIdx.x; inst < j.n_inst; inst += gridDim.x) {
+        const u64 base = (u64)inst * j.stride;
+        u32 hit = 0;
+        for (u32 i = threadIdx.x; i < j.n; i += blockDim.x) {
+            const u32 xf = arena[j.xf + base + i], xl = arena[j.xl + base + i];
+            hit |= (xl != 0u && xf != xl && arena[j.lw + base + i] != 0u);
+        }
+        if (__syncthreads_or((int)hit) && threadIdx.x == 0) flags[j.inst0 + inst] = 1u;
+    }
+}
+
+// K2c: fold the per-item site statistics of the block-parallel pass into the
+// per-launch table, skipping seed groups that the sequential pass re-runs.
+__global__ void __launch_bounds__(128) pg_stats_reduce(const PgWork* __restrict__ items, const u64* item_stats,
+                                                       const u32* flags, u64* launch_stats, u32 max_sites) {
+    const PgWork w = items[blockIdx.x];
+    __shared__ u32 s_skip;
+    if (threadIdx.x == 0) {
+        u32 f = 0;
+        for (u32 i = 0; i < w.nseeds; i++) f |= flags[w.inst0 + i];
+        s_skip = f;
+    }
+    __syncthreads();
+    if (s_skip) return;
+    const u64* src = item_stats + (u64)w.item * max_sites * 8u;
+    u64* dst = launch_stats + (u64)w.launch * max_sites * 8u;
+    for (u32 i = threadIdx.x; i < max_sites * 8u; i += blockDim.x) {
+        const u64 v = src[i];
+        if (!v) continue;
+        const u32 c = i & 7u;
+        if (c == 0) dst[i] = v;
+        else if (c == 3) atomicMax(&dst[i], v);
+        else atomicAdd(&dst[i], v);
+    }
+}
+
 __global__ void pg_reset_counters(long long* first_key, long long* counts) {
     const u32 i = threadIdx.x;
     if (i < 11) first_key[i] = 0x7FFFFFFFFFFFFFFFll;
@@ -238,6 +278,22 @@ cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 max_inst, const u32* aren
         dim3 g2((max_inst + 127) / 128, nj);
         pg_compare_fill<<<g2, 128, 0, st>>>(jobs + j0, arena_s, arena_t, input, slots, mm_key);
     }
+    return cudaGetLastError();
+}
+
+cudaError_t xb_detect(const PgXb* jobs, u32 n_jobs, u32 max_inst, const u32* arena, u32* flags, cudaStream_t st) {
+    for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
+        const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
+        dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
+        pg_xb_detect<<<grid, 256, 0, st>>>(jobs + j0, arena, flags);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t stats_reduce(const PgWork* items, u32 n_items, const u64* item_stats, const u32* flags, u64* launch_stats,
+                         u32 max_sites, cudaStream_t st) {
+    if (!n_items) return cudaSuccess;
+    pg_stats_reduce<<<n_items, 128, 0, st>>>(items, item_stats, flags, launch_stats, max_sites);
     return cudaGetLastError();
 }
 

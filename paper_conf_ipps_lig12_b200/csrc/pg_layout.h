@@ -51,13 +51,18 @@ struct PgLaunchK {
 
 struct PgWork {
     u32 launch;      // index into the launch table (and the record key)
-    u32 ngroups;     // instances in this CTA
-    u32 seed_j0;     // seed index of group 0
-    u32 seed_jstep;  // seed index stride between groups (= world)
-    u64 arena_off;   // u32-word offset of group 0's kernel arena
-    u64 input_off;   // u32-word offset of group 0's input region
-    u64 slot0;       // slot index (instance, this kernel, kind 0) of group 0
-    u64 slot_step;   // slot stride between groups
+    u32 ngroups;     // groups in this CTA = seeds x gb
+    u32 seed_j0;     // seed index of the item's seed 0
+    u32 seed_jstep;  // seed index stride between seeds (= world)
+    u32 blk0, blk1;  // emulated blocks [blk0, blk1) of every seed are processed by this CTA
+    u32 gb;          // block slots per seed: group g = seed (g / gb), block blk0 + i*gb + (g % gb)
+    u32 inst0;       // batch-local instance index of seed 0 (sequential-fallback flags)
+    u64 arena_off;   // u32-word offset of seed 0's kernel arena
+    u64 input_off;   // u32-word offset of seed 0's input region
+    u64 slot0;       // slot index (seed 0, this kernel, kind 0)
+    u64 slot_step;   // slot stride between seeds
+    u32 nseeds;      // seeds in this item
+    u32 item;        // item index (per-item site statistics)
 };
 
 struct PgSlot {
@@ -73,14 +78,16 @@ struct PgParams {
     const u32* input;
     PgSlot* slots;
     u64* counts;       // d_counts (int64[16] viewed as u64)
-    u64* site_stats;   // [n_launch][max_sites][8] for this kernel, or null
+    u64* site_stats;   // parallel pass: [item][max_sites][8]; sequential pass: [n_launch][max_sites][8]
+    u32* xb_flag;      // per batch-local instance: some global cell was shared between blocks
     u64 seed_base;
     u32 max_sites;
     u32 kernel_idx;
     u32 fuel;
+    u32 seq;           // 0: block-parallel pass; 1: sequential re-run of flagged seed groups
+    u32 input_mode, input_range, mask;
     u32 pad;
 };
-
 
 // K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive
 // instances of one launch (instance i at dst + i * stride, seed index j0 + i * jstep).
@@ -95,6 +102,15 @@ struct PgFill {
     u32 gid;      // PRF tag (X8)
     u32 value;    // PGF_CONST fill value
     u32 target;   // 0 arena (src), 1 arena (tgt), 2 input region
+};
+
+// K2b (pg_xb_detect) job: one global array written by a kernel, for n_inst
+// consecutive instances of one launch: flags instances whose cells were
+// accessed by two blocks with a committed write (X4 XB).
+struct PgXb {
+    u64 xf, xl, lw;   // u32-word offsets of instance 0 in the kernel arena
+    u64 stride;
+    u32 n, n_inst, inst0, pad;
 };
 
 // K3 (pg_compare) job: one compared global array for n_inst consecutive
