@@ -417,25 +417,48 @@ __device__ __noinline__ void pg_check(const PgC& C, PgT& t) {
 }
 
 // ------------------------------------------------------------------ records (H8)
-__device__ __noinline__ void pg_flush(const PgParams& P, PgT& t, u64 slot0) {
+// Each thread keeps its minimum event per kind; at the end of the CTA the lanes
+// of a warp that belong to the same instance merge theirs (lexicographic min by
+// successive warp-wide minima, counts by warp sum) and one lane updates the
+// (instance, kernel, kind) slot under its lock.  All 32 lanes call this.
+__device__ __noinline__ void pg_flush_warp(const PgParams& P, PgT& t, u32 valid, u64 slot0) {
     for (u32 k = 0; k < PG_NK; k++) {
-        if (!t.ecnt[k]) continue;
-        PgSlot* s = P.slots + slot0 + k;
-        atomicAdd(&s->count, (u64)t.ecnt[k]);
-        while (atomicCAS(&s->lock, 0u, 1u) != 0u) {
-        }
-        __threadfence();
-        volatile PgSlot* vs = s;
-        u32 cur[8];
+        u32 pending = valid && t.ecnt[k] != 0u;
+        for (;;) {
+            const u32 pm = __ballot_sync(PG_FULL, pending);
+            if (!pm) break;
+            const u32 leader = (u32)__ffs(pm) - 1u;
+            const u64 lslot = __shfl_sync(PG_FULL, slot0, leader);
+            u32 cand = pending && slot0 == lslot;
+            const u32 members = __ballot_sync(PG_FULL, cand);
+            const u32 cnt = __reduce_add_sync(PG_FULL, cand ? t.ecnt[k] : 0u);
+            u32 best[8];
 #pragma unroll
-        for (int i = 0; i < 8; i++) cur[i] = vs->f[i];
-        if (!vs->has || pg_lex_less(t.ebest[k], cur)) {
+            for (int f = 0; f < 8; f++) {
+                best[f] = __reduce_min_sync(PG_FULL, cand ? t.ebest[k][f] : PG_NEVER);
+                cand = cand && t.ebest[k][f] == best[f];
+            }
+            if (t.lane == leader) {
+                PgSlot* s = P.slots + lslot + k;
+                atomicAdd(&s->count, (u64)cnt);
+                while (atomicCAS(&s->lock, 0u, 1u) != 0u) {
+                }
+                __threadfence();
+                volatile PgSlot* vs = s;
+                u32 cur[8];
 #pragma unroll
-            for (int i = 0; i < 8; i++) vs->f[i] = t.ebest[k][i];
-            vs->has = 1u;
+                for (int i = 0; i < 8; i++) cur[i] = vs->f[i];
+                if (!vs->has || pg_lex_less(best, cur)) {
+#pragma unroll
+                    for (int i = 0; i < 8; i++) vs->f[i] = best[i];
+                    vs->has = 1u;
+                }
+                __threadfence();
+                atomicExch(&s->lock, 0u);
+            }
+            if (members & (1u << t.lane)) pending = 0u;
+            __syncwarp();
         }
-        __threadfence();
-        atomicExch(&s->lock, 0u);
     }
 }
 
@@ -671,7 +694,7 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
 #pragma unroll
     for (u32 v = 0; v < PG_VMAX; v++) {
         if (v >= V) break;
-        if (inst_ok && T[v].tlin < L.T) pg_flush(P, T[v], sW.slot0 + (u64)ms * sW.slot_step);
+        pg_flush_warp(P, T[v], inst_ok && T[v].tlin < L.T, sW.slot0 + (u64)ms * sW.slot_step);
     }
     if (!P.seq && inst_ok && tl0 == 0u) atomicAdd(&P.counts[0], s_inst[g]);
 #if PG_BANKCHK || PG_COALCHK
