@@ -1481,12 +1481,9 @@ struct Exec {
                 sowner[(size_t)A.local_index][c.addr] = {cur_block, cur_round, gw0};
             }
             if (!(cfg.checks & CHK_RACE)) continue;
-            if (w1 != w0) {   /* X16: site and val_b are those of the max-tid writer's last write */
-                int site1 = -1;
-                uint32_t v1 = val_of(w1, &site1);
-                event(K_RACE_WW, cur_round, rec_arr_id(c.arr), c.addr, gw0, cur_block * T + w1, (uint32_t)site1, v0,
-                      v1);
-            }
+            if (w1 != w0)   /* X16: (min writer, max writer), the committed write's site and value */
+                event(K_RACE_WW, cur_round, rec_arr_id(c.arr), c.addr, gw0, cur_block * T + w1, (uint32_t)site0, v0,
+                      0);
             auto rit = readers.find(c);
             if (rit != readers.end() && !rit->second.empty()) {
                 uint32_t rmin = *rit->second.begin(), rmax = *rit->second.rbegin();

@@ -42,6 +42,53 @@ struct Gen {
     };
     std::vector<std::string> preds;  // thread-dependent predicate variables, innermost last
     std::vector<Loop> loops;
+    std::vector<bool> log_;          // per array: a load may follow the thread's own store in one round
+
+    // ---------------------------------------------------------------- own-write analysis
+    // Conservative flow walk: which arrays may have been stored by this thread since
+    // the last barrier?  A load of such an array must consult the write log (X3);
+    // others read memory directly.
+    void lw_expr(const Node* n, const std::vector<bool>& stored) {
+        if (!n) return;
+        for (const Node* k : n->kids) lw_expr(k, stored);
+        if (n->kind == NK::Elem && stored[(size_t)n->ref]) log_[(size_t)n->ref] = true;
+    }
+    void lw_stmt(const Stmt* s, std::vector<bool>& st) {
+        if (!s) return;
+        switch (s->kind) {
+        case SK::Seq:
+            for (const Stmt* c : s->seq) lw_stmt(c, st);
+            break;
+        case SK::Assign: lw_expr(s->value, st); break;
+        case SK::Store:
+            for (const Node* i : s->index) lw_expr(i, st);
+            lw_expr(s->value, st);
+            st[(size_t)s->arr] = true;
+            break;
+        case SK::Sync: std::fill(st.begin(), st.end(), false); break;
+        case SK::If: {
+            lw_expr(s->cond, st);
+            std::vector<bool> a = st, b = st;
+            lw_stmt(s->body, a);
+            lw_stmt(s->other, b);
+            for (size_t i = 0; i < st.size(); i++) st[i] = a[i] || b[i];
+            break;
+        }
+        case SK::Loop: {
+            lw_stmt(s->init, st);
+            for (int pass = 0; pass < 3; pass++) {  // a store can reach a load of the next iteration
+                std::vector<bool> in = st;
+                lw_expr(s->cond, in);
+                lw_stmt(s->body, in);
+                lw_stmt(s->step, in);
+                for (size_t i = 0; i < st.size(); i++) st[i] = st[i] || in[i];
+            }
+            lw_expr(s->cond, st);
+            break;
+        }
+        default: break;
+        }
+    }
 
     Gen(const Kernel& k, const CodegenOptions& o) : K(k), O(o) {
         mask = o.bits >= 32 ? 0xFFFFFFFFu : ((1u << o.bits) - 1u);
@@ -76,7 +123,7 @@ struct Gen {
         for (size_t k = 1; k < iv.size(); k++) {
             std::string dim;
             if (a.space == PRIVATE) dim = hex(a.dims[k]->lit);
-            else dim = "C.L->arr[" + std::to_string(arr) + "].d" + std::to_string(k);
+            else dim = "pg_sL.arr[" + std::to_string(arr) + "].d" + std::to_string(k);
             line(f + " = " + f + " * " + dim + " + " + iv[k] + ";");
         }
         return f;
@@ -90,8 +137,8 @@ struct Gen {
             std::string src;
             if (n->ref < 3) src = "t.tid[" + std::to_string(c) + "]";
             else if (n->ref < 6) src = "t.bid[" + std::to_string(c) + "]";
-            else if (n->ref < 9) src = "C.L->bdim[" + std::to_string(c) + "]";
-            else src = "C.L->gdim[" + std::to_string(c) + "]";
+            else if (n->ref < 9) src = "pg_sL.bdim[" + std::to_string(c) + "]";
+            else src = "pg_sL.gdim[" + std::to_string(c) + "]";
             return "pg_m(" + src + ")";
         }
         case NK::Elem: {
@@ -100,16 +147,16 @@ struct Gen {
             std::string r = tmp();
             std::string A = std::to_string(n->ref), S = std::to_string(n->site) + "u";
             if (a.space == SHARED) {
-                line("u32 " + r + " = pg_ld_sh<" + A + ", " + (reader_tracked(n->ref) ? "true" : "false") +
-                     ">(C, t, ss, " + pr + ", " + f + ", " + S + ");");
+                line("u32 " + r + " = pg_ld_sh<" + A + ", " + (reader_tracked(n->ref) ? "true" : "false") + ", " +
+                     (log_[(size_t)n->ref] ? "true" : "false") + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
             } else if (a.space == GLOBAL) {
                 if (a.written)
-                    line("u32 " + r + " = pg_ld_gt<" + A + ", " + (reader_tracked(n->ref) ? "true" : "false") +
-                         ">(C, t, ss, " + pr + ", " + f + ", " + S + ");");
+                    line("u32 " + r + " = pg_ld_gt<" + A + ", " + (reader_tracked(n->ref) ? "true" : "false") + ", " +
+                         (log_[(size_t)n->ref] ? "true" : "false") + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
                 else
-                    line("u32 " + r + " = pg_ld_gi<" + A + ">(C, t, ss, " + pr + ", " + f + ", " + S + ");");
+                    line("u32 " + r + " = pg_ld_gi<" + A + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
             } else {
-                line("u32 " + r + " = pg_priv_ok(C, t, " + pr + ", " + f + ", " + hex(priv_size(a)) + ", " +
+                line("u32 " + r + " = pg_priv_ok(C, t, c, " + pr + ", " + f + ", " + hex(priv_size(a)) + ", " +
                      hex(0x200u + (uint32_t)a.slot) + ", " + S + ", 0u, 0u) ? F.p" + std::to_string(a.slot) + "[" +
                      f + "] : 0u;");
             }
@@ -204,10 +251,10 @@ struct Gen {
             std::string f = flat_index(&tmpn, s->arr, pe);
             std::string v = ex(s->value, pe);
             std::string A = std::to_string(s->arr), S = std::to_string(s->site) + "u";
-            if (a.space == SHARED) line("pg_st_sh<" + A + ">(C, t, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
-            else if (a.space == GLOBAL) line("pg_st_gt<" + A + ">(C, t, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
+            if (a.space == SHARED) line("pg_st_sh<" + A + ">(C, t, c, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
+            else if (a.space == GLOBAL) line("pg_st_gt<" + A + ">(C, t, c, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
             else
-                line("if (pg_priv_ok(C, t, " + pe + ", " + f + ", " + hex(priv_size(a)) + ", " +
+                line("if (pg_priv_ok(C, t, c, " + pe + ", " + f + ", " + hex(priv_size(a)) + ", " +
                      hex(0x200u + (uint32_t)a.slot) + ", " + S + ", " + v + ", 1u)) F.p" + std::to_string(a.slot) +
                      "[" + f + "] = " + v + ";");
             line("}");
@@ -315,7 +362,7 @@ struct Gen {
         body << "L" << L.cont_label << ":;\n";
         if (s->step) stmt(s->step);
         loops.pop_back();
-        line("pg_tick(C, t, t.live);");
+        line("pg_tick(C, t, c, t.live);");
         line("if (++C.ufuel > C.fuel) { t.live = 0u; return PG_END; }");
         line("goto L" + std::to_string(head) + ";");
         body << "L" << L.exit_label << ":;\n";
@@ -352,12 +399,17 @@ struct Gen {
             stmt(s->step);
             preds.pop_back();
         }
-        line("pg_tick(C, t, " + L.act + " & t.live);");
+        line("pg_tick(C, t, c, " + L.act + " & t.live);");
         line("}");
         line("}");
     }
 
     std::string run() {
+        log_.assign(K.arrays.size(), false);
+        {
+            std::vector<bool> st(K.arrays.size(), false);
+            lw_stmt(K.body, st);
+        }
         stmt(K.body);
         line("t.live = 0u; return PG_END;");
         std::ostringstream o;
@@ -381,12 +433,30 @@ struct Gen {
         o << "  static __device__ __forceinline__ void init(Frame& F, const PgC& C, PgT& t) {\n";
         for (size_t i = 0; i < K.vars.size(); i++) {
             if (K.vars[i].scalar)
-                o << "    F.v" << i << " = pg_m((u32)C.L->scal[" << K.vars[i].scalar_index << "]);\n";
+                o << "    F.v" << i << " = pg_m((u32)pg_sL.scal[" << K.vars[i].scalar_index << "]);\n";
             else
                 o << "    F.v" << i << " = 0u;\n";
         }
         o << "  }\n";
-        o << "  static __device__ __forceinline__ u32 seg(Frame& F, PgC& C, PgT& t, u64* ss, u32 resume) {\n";
+        // per-array claim / check dispatch for the write log (array kind fixed at code-generation time)
+        for (int phase = 0; phase < 2; phase++) {
+            o << "  static __device__ __forceinline__ void " << (phase ? "check" : "claim")
+              << "(const PgC& C, const PgT& t, PgCold& c) {\n";
+            o << "    for (u32 i = 0; i < t.nlog; i++) {\n      const u32 cell = c.lcell[i], flat = cell & 0xFFFFFFu;\n";
+            o << "      switch (cell >> 24) {\n";
+            for (size_t a = 0; a < K.arrays.size(); a++) {
+                const ArrayDecl& A = K.arrays[a];
+                if (!A.written || A.space == PRIVATE) continue;
+                const char* sp = A.space == SHARED ? "sh" : "gt";
+                if (phase == 0)
+                    o << "        case " << a << ": pg_claim_" << sp << "<" << a << ">(C, t, flat); break;\n";
+                else
+                    o << "        case " << a << ": pg_check_" << sp << "<" << a << ", "
+                      << (reader_tracked((int)a) ? "true" : "false") << ">(C, t, c, i, flat); break;\n";
+            }
+            o << "        default: break;\n      }\n    }\n  }\n";
+        }
+        o << "  static __device__ __forceinline__ u32 seg(Frame& F, PgC& C, PgT& t, PgCold& c, u64* ss, u32 resume) {\n";
         o << "    switch (resume) {\n      case 0u: goto R0;\n";
         for (int k = 1; k <= nsync; k++) o << "      case " << k << "u: goto R" << k << ";\n";
         o << "      default: return PG_END;\n    }\n";

@@ -30,19 +30,13 @@ __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ 
         const u64 seed = seed_base + (u64)f.j0 + (u64)inst * f.jstep;
         if (f.op == PGF_CONST) {
             for (u32 i = threadIdx.x; i < f.n; i += blockDim.x) base[i] = f.value;
-        } else if (f.op == PGF_INPUT) {
+        } else {  // PGF_INPUT (initial values of an input region or of a written array)
             for (u32 i = threadIdx.x; i < f.n; i += blockDim.x) base[i] = init_value(mode, range, mask, seed, f.gid, i);
-        } else {
-            u64* cells = (u64*)base;
-            for (u32 i = threadIdx.x; i < f.n; i += blockDim.x)
-                cells[i] = ((u64)PG_NEVER << 32) | init_value(mode, range, mask, seed, f.gid, i);
         }
     }
 }
 
-__device__ __forceinline__ u32 cmp_val(const u32* region, u32 kind, u64 off, u32 i) {
-    return kind == 0 ? (u32)((const u64*)(region + off))[i] : region[off + i];
-}
+__device__ __forceinline__ u32 cmp_val(const u32* region, u32 kind, u64 off, u32 i) { return region[off + i]; }
 
 // K3a: count mismatching cells per (instance, array); keep the minimum (gid, addr)
 // per instance.

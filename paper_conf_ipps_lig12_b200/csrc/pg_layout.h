@@ -27,15 +27,17 @@ struct PgArr {
     u32 kind;       // PGA_*
     u32 rec_id;     // array id in records: gid | 0x100 + slot | 0x200 + slot
     u32 gid;        // pair-level global id (PRF tag, X8)
-    u32 smem_cells; // shared: byte offset of u64 cells in the group region
-    u32 smem_wmax;  // shared: byte offset of u32 wmax stamps
-    u32 smem_rmin, smem_rmax;
     u32 flags;      // bit0: reader stamps present (array read and written, race checks on)
+    // shared arrays: byte offsets in the group's shared region
+    u32 s_val, s_own, s_wmax, s_rmin, s_rmax;
     u32 pad;
-    u64 off_cells;  // global tracked: u32-word offset of u64 cells in the instance arena
-    u64 off_lw;     // last committing writer (gtid + 1)
-    u64 off_wmax, off_rmin, off_rmax, off_xf, off_xl;
-    u64 off_in;     // global input: u32-word offset in the instance input region
+    // global arrays written by the kernel: u32-word offsets in the instance arena
+    u64 off_val;    // values
+    u64 off_own;    // owner stamp of the last commit: ((2^20-1 - step) << 12) | tid
+    u64 off_lw;     // last committing writer (gtid + 1; 0 = initial)
+    u64 off_wmax, off_rmin, off_rmax;   // race stamps (~0: absent)
+    u64 off_xf, off_xl;                 // first / last accessing block + 1 (~0: absent)
+    u64 off_in;     // global arrays the kernel only reads: u32-word offset in the input region
 };
 
 struct PgLaunchK {
@@ -43,8 +45,8 @@ struct PgLaunchK {
     i32 scal[8];
     u32 T, nblocks;
     u32 lpg, gpw, wpg, V, P, cta_threads;
-    u32 smem_group_bytes, smem_cells_bytes;  // per group: cells region first, then u32 stamps
-    u32 n_arrays, smem_never_off;             // stamps in [cells_bytes, never_off) start at 0, the rest at ~0
+    // per-group shared region: [values | stamps starting at 0 | stamps starting at ~0]
+    u32 smem_group_bytes, smem_zero_off, smem_never_off, n_arrays;
     u64 arena_stride, input_stride;          // u32 words per instance
     PgArr arr[PG_MAXARR];
 };
@@ -116,7 +118,7 @@ struct PgXb {
 // K3 (pg_compare) job: one compared global array for n_inst consecutive
 // instances of one launch (H7).
 struct PgCmp {
-    u64 src_off, tgt_off;        // u32-word offsets of instance 0: u64 cells in an arena (kind 0) or u32 input (kind 1)
+    u64 src_off, tgt_off;        // u32-word offsets of instance 0: values in an arena (kind 0) or the input (kind 1)
     u64 src_stride, tgt_stride;  // per-instance strides of the regions the offsets point into
     u64 src_lw, tgt_lw;          // last-writer words of instance 0 (kind 0 only)
     u64 slot0, slot_step;        // MISMATCH slot of (instance 0, kernel 0) and stride
