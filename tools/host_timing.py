@@ -28,4 +28,4 @@ for it in range(3):
         t = r.timing()
         print("%-28s host %7.1f ms  device total %7.1f ms  K2 %7.1f ms  launches %d" %
               (name, 1e3 * h, t["ms_total"], t["ms_eval"], t["launches"]))
-    print("iteration %d wall %.1f ms" % (it, 1e3 * wall))
+    print("iteration %d wall %.1f ms" % (it, 1e3 * wall), flush=True)
