@@ -439,23 +439,25 @@ struct Gen {
         }
         o << "  }\n";
         // per-array claim / check dispatch for the write log (array kind fixed at code-generation time)
-        for (int phase = 0; phase < 2; phase++) {
-            o << "  static __device__ __forceinline__ void " << (phase ? "check" : "claim")
-              << "(const PgC& C, const PgT& t, PgCold& c) {\n";
-            o << "    for (u32 i = 0; i < t.nlog; i++) {\n      const u32 cell = c.lcell[i], flat = cell & 0xFFFFFFu;\n";
-            o << "      switch (cell >> 24) {\n";
-            for (size_t a = 0; a < K.arrays.size(); a++) {
-                const ArrayDecl& A = K.arrays[a];
-                if (!A.written || A.space == PRIVATE) continue;
-                const char* sp = A.space == SHARED ? "sh" : "gt";
-                if (phase == 0)
-                    o << "        case " << a << ": pg_claim_" << sp << "<" << a << ">(C, t, flat); break;\n";
-                else
-                    o << "        case " << a << ": pg_check_" << sp << "<" << a << ", "
-                      << (reader_tracked((int)a) ? "true" : "false") << ">(C, t, c, i, flat); break;\n";
-            }
-            o << "        default: break;\n      }\n    }\n  }\n";
+        o << "  static __device__ __forceinline__ void claim_one(const PgC& C, const PgT& t, u32 cell) {\n";
+        o << "    const u32 flat = cell & 0xFFFFFFu;\n    switch (cell >> 24) {\n";
+        for (size_t a = 0; a < K.arrays.size(); a++) {
+            const ArrayDecl& A = K.arrays[a];
+            if (!A.written || A.space == PRIVATE) continue;
+            o << "      case " << a << ": pg_claim_" << (A.space == SHARED ? "sh" : "gt") << "<" << a
+              << ">(C, t, flat); break;\n";
         }
+        o << "      default: break;\n    }\n  }\n";
+        o << "  static __device__ __forceinline__ void check_one(const PgC& C, const PgT& t, PgCold& c, u32 cell, "
+             "u32 val, u32 site) {\n";
+        o << "    const u32 flat = cell & 0xFFFFFFu;\n    switch (cell >> 24) {\n";
+        for (size_t a = 0; a < K.arrays.size(); a++) {
+            const ArrayDecl& A = K.arrays[a];
+            if (!A.written || A.space == PRIVATE) continue;
+            o << "      case " << a << ": pg_check_" << (A.space == SHARED ? "sh" : "gt") << "<" << a << ", "
+              << (reader_tracked((int)a) ? "true" : "false") << ">(C, t, c, flat, val, site); break;\n";
+        }
+        o << "      default: break;\n    }\n  }\n";
         o << "  static __device__ __forceinline__ u32 seg(Frame& F, PgC& C, PgT& t, PgCold& c, u64* ss, u32 resume) {\n";
         o << "    switch (resume) {\n      case 0u: goto R0;\n";
         for (int k = 1; k <= nsync; k++) o << "      case " << k << "u: goto R" << k << ";\n";

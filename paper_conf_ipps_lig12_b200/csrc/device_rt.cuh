@@ -83,6 +83,7 @@ struct PgT {        // hot per-emulated-thread state (kept in registers)
     u32 tlin, gtid;
     u32 lane, ekey; // HW lane; emulated-warp key within the HW warp (63: idle)
     u32 nlog;
+    u32 l0cell, l0val, l0site;  // write-log entry 0 (registers; entries 1.. live in PgCold)
     u32 fuel;
     u32 sg;         // byte offset of this instance's shared region in pg_dsmem
     u64 seed;
@@ -91,7 +92,7 @@ struct PgT {        // hot per-emulated-thread state (kept in registers)
 };
 
 struct PgCold {     // per-emulated-thread state that lives in local memory
-    u32 lcell[PG_WMAX];   // write log (X3): cell id = array << 24 | flat
+    u32 lcell[PG_WMAX];   // write log entries 1.. (X3): cell id = array << 24 | flat
     u32 lval[PG_WMAX];
     u16 lsite[PG_WMAX];
     u32 ecnt[PG_NK];      // events per kind
@@ -183,7 +184,12 @@ __device__ __noinline__ void pg_coal_global(u32 round, u32 lane, u32 ekey, u32 g
 
 // ------------------------------------------------------------------ loads / stores
 __device__ __forceinline__ u32 pg_log_find(const PgT& t, const PgCold& c, u32 cell, u32& v) {
-    for (u32 i = 0; i < t.nlog; i++)
+    if (t.nlog == 0u) return 0u;
+    if (t.l0cell == cell) {
+        v = t.l0val;
+        return 1u;
+    }
+    for (u32 i = 1; i < t.nlog; i++)
         if (c.lcell[i] == cell) {
             v = c.lval[i];
             return 1u;
@@ -191,9 +197,9 @@ __device__ __forceinline__ u32 pg_log_find(const PgT& t, const PgCold& c, u32 ce
     return 0u;
 }
 
-__device__ __noinline__ void pg_log_write(u32 round, u32 gtid, u32& nlog, PgCold& c, u32 cell, u32 val, u32 site,
-                                          u32 rec, u32 flat) {
-    for (u32 i = 0; i < nlog; i++) {
+__device__ __noinline__ void pg_log_write_slow(u32 round, u32 gtid, u32& nlog, PgCold& c, u32 cell, u32 val, u32 site,
+                                               u32 rec, u32 flat) {
+    for (u32 i = 1; i < nlog; i++) {
         if (c.lcell[i] == cell) {
             c.lval[i] = val;
             c.lsite[i] = (u16)site;
@@ -208,6 +214,21 @@ __device__ __noinline__ void pg_log_write(u32 round, u32 gtid, u32& nlog, PgCold
     c.lval[nlog] = val;
     c.lsite[nlog] = (u16)site;
     nlog++;
+}
+
+__device__ __forceinline__ void pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell, u32 val, u32 site, u32 rec,
+                                             u32 flat) {
+    if (t.nlog == 0u) {
+        t.l0cell = cell;
+        t.l0val = val;
+        t.l0site = site;
+        t.nlog = 1u;
+    } else if (t.l0cell == cell) {
+        t.l0val = val;
+        t.l0site = site;
+    } else {
+        pg_log_write_slow(C.round, t.gtid, t.nlog, c, cell, val, site, rec, flat);
+    }
 }
 
 __device__ __forceinline__ u32 pg_poison_sh(const PgT& t, u32 rec, u32 flat) {
@@ -232,7 +253,7 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
         return pv;
     }
 #if PG_RACECHK
-    if (RD) {
+    if (RD && pg_sL.T > 1u) {
         atomicMin(pg_sh(t, PG_ARR(A).s_rmin) + flat, pg_stamp_min(C, t));
         atomicMax(pg_sh(t, PG_ARR(A).s_rmax) + flat, pg_stamp_max(C, t));
     }
@@ -263,7 +284,7 @@ __device__ __forceinline__ void pg_st_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32
 #endif
         return;
     }
-    pg_log_write(C.round, t.gtid, t.nlog, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+    pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
 }
 
 // XB bookkeeping (X4): first and last block that accessed a global cell.  Kept
@@ -294,7 +315,7 @@ __device__ __forceinline__ u32 pg_ld_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
     }
     pg_xb_mark<A>(t, flat);
 #if PG_RACECHK
-    if (RD) {
+    if (RD && pg_sL.T > 1u) {
         atomicMin(t.arena + PG_ARR(A).off_rmin + flat, pg_stamp_min(C, t));
         atomicMax(t.arena + PG_ARR(A).off_rmax + flat, pg_stamp_max(C, t));
     }
@@ -318,7 +339,7 @@ __device__ __forceinline__ void pg_st_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32
         return;
     }
     pg_xb_mark<A>(t, flat);
-    pg_log_write(C.round, t.gtid, t.nlog, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+    pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
 }
 
 // Global array this kernel only reads: the instance's input region.
@@ -367,23 +388,22 @@ template <int A>
 __device__ __forceinline__ void pg_claim_sh(const PgC& C, const PgT& t, u32 flat) {
     atomicMin(pg_sh(t, PG_ARR(A).s_own) + flat, pg_stamp_min(C, t));
 #if PG_RACECHK
-    atomicMax(pg_sh(t, PG_ARR(A).s_wmax) + flat, pg_stamp_max(C, t));
+    if (pg_sL.T > 1u) atomicMax(pg_sh(t, PG_ARR(A).s_wmax) + flat, pg_stamp_max(C, t));
 #endif
 }
 template <int A>
 __device__ __forceinline__ void pg_claim_gt(const PgC& C, const PgT& t, u32 flat) {
     atomicMin(t.arena + PG_ARR(A).off_own + flat, pg_stamp_min(C, t));
 #if PG_RACECHK
-    atomicMax(t.arena + PG_ARR(A).off_wmax + flat, pg_stamp_max(C, t));
+    if (pg_sL.T > 1u) atomicMax(t.arena + PG_ARR(A).off_wmax + flat, pg_stamp_max(C, t));
 #endif
 }
 
-__device__ __noinline__ void pg_race_check(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 i, u32 rec,
-                                           u32 flat, u32 own, u32 wmax, u32 has_readers, u32 rmin, u32 rmax) {
+__device__ __noinline__ void pg_race_check(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 val, u32 site,
+                                           u32 rec, u32 flat, u32 own, u32 wmax, u32 has_readers, u32 rmin, u32 rmax) {
     const u32 base = gtid - tlin;
     const u32 w0 = own & 0xFFFu, w1 = wmax & 0xFFFu;
-    if (w1 != w0 && tlin == w0)
-        pg_event(c, PGK_WW, round, rec, flat, gtid, base + w1, c.lsite[i], c.lval[i], 0);
+    if (w1 != w0 && tlin == w0) pg_event(c, PGK_WW, round, rec, flat, gtid, base + w1, site, val, 0);
     if (has_readers && (rmax >> 12) == step) {
         const u32 r0 = rmin & 0xFFFu, r1 = rmax & 0xFFFu;
         if (!(r0 == r1 && w0 == w1 && r0 == w0)) {
@@ -391,38 +411,57 @@ __device__ __noinline__ void pg_race_check(u32 round, u32 step, u32 tlin, u32 gt
             if (r0 != w0) { ta = w0; tb = r0; }
             else if (r1 != w0) { ta = w0; tb = r1; }
             else { ta = w1; tb = r0; }
-            if (tlin == ta) pg_event(c, PGK_RW, round, rec, flat, base + ta, base + tb, c.lsite[i], c.lval[i], 0);
+            if (tlin == ta) pg_event(c, PGK_RW, round, rec, flat, base + ta, base + tb, site, val, 0);
         }
     }
 }
 
 template <int A, bool RD>
-__device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& c, u32 i, u32 flat) {
+__device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
     const u32 own = pg_sh(t, PG_ARR(A).s_own)[flat];
-    if (own == pg_stamp_min(C, t)) pg_sh(t, PG_ARR(A).s_val)[flat] = c.lval[i];
+    if (own == pg_stamp_min(C, t)) pg_sh(t, PG_ARR(A).s_val)[flat] = val;
 #if PG_RACECHK
-    const u32 wmax = pg_sh(t, PG_ARR(A).s_wmax)[flat];
-    const u32 rmin = RD ? pg_sh(t, PG_ARR(A).s_rmin)[flat] : 0u;
-    const u32 rmax = RD ? pg_sh(t, PG_ARR(A).s_rmax)[flat] : 0u;
-    if ((wmax & 0xFFFu) != (own & 0xFFFu) || (RD && (rmax >> 12) == C.step))
-        pg_race_check(C.round, C.step, t.tlin, t.gtid, c, i, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin, rmax);
+    if (pg_sL.T > 1u) {
+        const u32 wmax = pg_sh(t, PG_ARR(A).s_wmax)[flat];
+        const u32 rmin = RD ? pg_sh(t, PG_ARR(A).s_rmin)[flat] : 0u;
+        const u32 rmax = RD ? pg_sh(t, PG_ARR(A).s_rmax)[flat] : 0u;
+        if ((wmax & 0xFFFu) != (own & 0xFFFu) || (RD && (rmax >> 12) == C.step))
+            pg_race_check(C.round, C.step, t.tlin, t.gtid, c, val, site, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin,
+                          rmax);
+    }
 #endif
 }
 
 template <int A, bool RD>
-__device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& c, u32 i, u32 flat) {
+__device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
     const u32 own = t.arena[PG_ARR(A).off_own + flat];
     if (own == pg_stamp_min(C, t)) {
-        t.arena[PG_ARR(A).off_val + flat] = c.lval[i];
+        t.arena[PG_ARR(A).off_val + flat] = val;
         t.arena[PG_ARR(A).off_lw + flat] = t.gtid + 1u;
     }
 #if PG_RACECHK
-    const u32 wmax = t.arena[PG_ARR(A).off_wmax + flat];
-    const u32 rmin = RD ? t.arena[PG_ARR(A).off_rmin + flat] : 0u;
-    const u32 rmax = RD ? t.arena[PG_ARR(A).off_rmax + flat] : 0u;
-    if ((wmax & 0xFFFu) != (own & 0xFFFu) || (RD && (rmax >> 12) == C.step))
-        pg_race_check(C.round, C.step, t.tlin, t.gtid, c, i, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin, rmax);
+    if (pg_sL.T > 1u) {
+        const u32 wmax = t.arena[PG_ARR(A).off_wmax + flat];
+        const u32 rmin = RD ? t.arena[PG_ARR(A).off_rmin + flat] : 0u;
+        const u32 rmax = RD ? t.arena[PG_ARR(A).off_rmax + flat] : 0u;
+        if ((wmax & 0xFFFu) != (own & 0xFFFu) || (RD && (rmax >> 12) == C.step))
+            pg_race_check(C.round, C.step, t.tlin, t.gtid, c, val, site, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin,
+                          rmax);
+    }
 #endif
+}
+
+template <class K>
+__device__ __forceinline__ void pg_claim_all(const PgC& C, const PgT& t, const PgCold& c) {
+    if (t.nlog == 0u) return;
+    K::claim_one(C, t, t.l0cell);
+    for (u32 i = 1; i < t.nlog; i++) K::claim_one(C, t, c.lcell[i]);
+}
+template <class K>
+__device__ __forceinline__ void pg_check_all(const PgC& C, const PgT& t, PgCold& c) {
+    if (t.nlog == 0u) return;
+    K::check_one(C, t, c, t.l0cell, t.l0val, t.l0site);
+    for (u32 i = 1; i < t.nlog; i++) K::check_one(C, t, c, c.lcell[i], c.lval[i], c.lsite[i]);
 }
 
 // ------------------------------------------------------------------ records (H8)
@@ -541,44 +580,48 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         __syncthreads();
     }
     const u32 gbytes = pg_sL.smem_group_bytes;
+    const u32 T_ = pg_sL.T;
+    const bool warp_blocks = T_ <= 32u;  // an emulated block never spans warps: warp-level barriers suffice
     u64* sstats = (u64*)(pg_dsmem + (u64)pg_sL.P * gbytes);
-    u32* s_alive = (u32*)(sstats + ((PG_BANKCHK || PG_COALCHK) ? PG_NSTATS * 8 : 0));
-    u32* s_alive_next = s_alive + pg_sL.P;
-    u32* s_rounds = s_alive_next + pg_sL.P;
-    u64* s_inst = (u64*)(((unsigned long long)(s_rounds + pg_sL.P) + 7) & ~7ull);
+    u32* s_grounds = (u32*)(sstats + ((PG_BANKCHK || PG_COALCHK) ? PG_NSTATS * 8 : 0));  // per group (T > 32)
     // shared regions: initialised once per CTA (stamps are step-tagged)
-    for (u32 gi = 0; gi < G; gi++) {
-        u32* z = (u32*)(pg_dsmem + (u64)gi * gbytes + pg_sL.smem_zero_off);
+    {
         const u32 zw = (pg_sL.smem_never_off - pg_sL.smem_zero_off) / 4u;
-        for (u32 i = threadIdx.x; i < zw; i += blockDim.x) z[i] = 0u;
-        u32* nv = (u32*)(pg_dsmem + (u64)gi * gbytes + pg_sL.smem_never_off);
         const u32 nw = (gbytes - pg_sL.smem_never_off) / 4u;
-        for (u32 i = threadIdx.x; i < nw; i += blockDim.x) nv[i] = PG_NEVER;
+        const u32 per = zw + nw;
+        for (u32 i = threadIdx.x; i < G * per; i += blockDim.x) {
+            const u32 gi = i / per, j = i - gi * per;
+            u32* base = (u32*)(pg_dsmem + (u64)gi * gbytes + pg_sL.smem_zero_off);
+            base[j] = j < zw ? 0u : PG_NEVER;
+        }
     }
 #if PG_BANKCHK || PG_COALCHK
     for (u32 i = threadIdx.x; i < PG_NSTATS * 8; i += blockDim.x) sstats[i] = 0;
 #else
     sstats = nullptr;
 #endif
-    for (u32 i = threadIdx.x; i < pg_sL.P; i += blockDim.x) { s_inst[i] = 0; s_alive_next[i] = 0; }
+    for (u32 i = threadIdx.x; i < pg_sL.P; i += blockDim.x) s_grounds[i] = 0;
 
     PgC C;
     C.step = 0;
     C.fuel = P.fuel;
-    const u32 T_ = pg_sL.T;
     const u32 lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-    u32 g, tl0, lane_ok, ekey;
-    if (T_ <= 32u) {
+    u32 g, tl0, lane_ok, ekey, gmask;
+    if (warp_blocks) {
         const u32 sub = lane / T_;
         g = warp * pg_sL.gpw + sub;
         tl0 = lane - sub * T_;
         lane_ok = sub < pg_sL.gpw;
         ekey = lane_ok ? sub : 63u;
+        const u32 span = pg_sL.gpw * T_;
+        gmask = lane_ok ? (T_ == 32u ? PG_FULL : (((1u << T_) - 1u) << (sub * T_)))
+                        : (span >= 32u ? 0u : ~((1u << span) - 1u));
     } else {
         g = warp / pg_sL.wpg;
         tl0 = (warp % pg_sL.wpg) * 32u + lane;
         lane_ok = 1u;
         ekey = 0u;
+        gmask = PG_FULL;
     }
     const u32 inst_ok = lane_ok && g < G;
     const u32 gc = inst_ok ? g : 0u;
@@ -602,27 +645,32 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         t.arena = P.arena + pg_sW.arena_off + (u64)ms * pg_sL.arena_stride;
         t.input = P.input + pg_sW.input_off + (u64)ms * pg_sL.input_stride;
         t.sg = gc * gbytes;
+        t.l0cell = t.l0val = t.l0site = 0u;
         for (u32 k = 0; k < PG_NK; k++) Cd[v].ecnt[k] = 0;
         t.live = ok;
     }
+    __syncthreads();
+    const bool grid_1d = pg_sL.gdim[1] == 1u && pg_sL.gdim[2] == 1u;
+    u64 inst = 0;  // instances of this group (accumulated by its lane tl0 == 0)
     const u32 nsteps = (pg_sW.blk1 - pg_sW.blk0 + GB - 1) / GB;
     for (u32 st = 0; st < nsteps; st++) {
         const u32 blk = pg_sW.blk0 + st * GB + bs;
         const u32 blk_ok = blk < pg_sW.blk1;
-        for (u32 i = threadIdx.x; i < pg_sL.P; i += blockDim.x) {
-            s_alive[i] = i < G && pg_sW.blk0 + st * GB + (i % GB) < pg_sW.blk1;
-            s_rounds[i] = 0;
-        }
-        __syncthreads();
         C.step0 = C.step + 1u;
+        u32 alive_rounds = 0;  // rounds this thread entered alive (X19: group rounds = max over threads)
 #pragma unroll
         for (u32 v = 0; v < PG_VMAX; v++) {
             if (v >= V) break;
             PgT& t = T[v];
             t.blk = blk;
-            t.bid[0] = blk % pg_sL.gdim[0];
-            t.bid[1] = (blk / pg_sL.gdim[0]) % pg_sL.gdim[1];
-            t.bid[2] = blk / (pg_sL.gdim[0] * pg_sL.gdim[1]);
+            if (grid_1d) {
+                t.bid[0] = blk;
+                t.bid[1] = t.bid[2] = 0u;
+            } else {
+                t.bid[0] = blk % pg_sL.gdim[0];
+                t.bid[1] = (blk / pg_sL.gdim[0]) % pg_sL.gdim[1];
+                t.bid[2] = blk / (pg_sL.gdim[0] * pg_sL.gdim[1]);
+            }
             t.live = inst_ok && t.tlin < T_ && blk_ok;
             t.gtid = blk * T_ + t.tlin;
             K::init(F[v], C, t);
@@ -633,40 +681,48 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
             C.step++;
             C.ufuel = 0;
             u32 r = PG_END;
+            u32 any_start = 0;
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
+                any_start |= T[v].live;
                 T[v].nlog = 0;
                 T[v].fuel = 0;
                 r = K::seg(F[v], C, T[v], Cd[v], sstats, resume);
             }
-            __syncthreads();
+            alive_rounds += any_start;
+            if (warp_blocks) __syncwarp(); else __syncthreads();
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
-                K::claim(C, T[v], Cd[v]);
+                pg_claim_all<K>(C, T[v], Cd[v]);
             }
-            __syncthreads();
+            if (warp_blocks) __syncwarp(); else __syncthreads();
             u32 any = 0;
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
-                K::check(C, T[v], Cd[v]);
+                pg_check_all<K>(C, T[v], Cd[v]);
                 any |= T[v].live;
             }
-            if (any && inst_ok) s_alive_next[g] = 1u;
-            __syncthreads();
-            for (u32 i = threadIdx.x; i < G; i += blockDim.x) {
-                s_rounds[i] += s_alive[i];
-                s_alive[i] = s_alive_next[i];
-                s_alive_next[i] = 0u;
-            }
             C.round++;
-            const int more = __syncthreads_or((int)any);
+            const int more = warp_blocks ? __any_sync(PG_FULL, any) : __syncthreads_or((int)any);
             if (r == PG_END || !more) break;
             resume = r;
         }
-        for (u32 i = threadIdx.x; i < G; i += blockDim.x) s_inst[i] += (u64)T_ * s_rounds[i];
+        // rounds of this group's block = max over its threads of the rounds they entered alive
+        u32 grounds;
+        if (warp_blocks) {
+            grounds = __reduce_max_sync(PG_FULL, 0u);  // keep the warp converged before the segmented max
+            grounds = gmask ? __reduce_max_sync(gmask, alive_rounds) : 0u;
+        } else {
+            if (inst_ok && alive_rounds) atomicMax(&s_grounds[g], alive_rounds);
+            __syncthreads();
+            grounds = inst_ok ? s_grounds[g] : 0u;
+            __syncthreads();
+            if (inst_ok && tl0 == 0u) s_grounds[g] = 0u;
+        }
+        inst += (u64)T_ * grounds;
     }
     __syncthreads();
 #if PG_RACECHK
@@ -697,7 +753,7 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         if (v >= V) break;
         pg_flush_warp(P, lane, Cd[v], inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)ms * pg_sW.slot_step);
     }
-    if (!P.seq && inst_ok && tl0 == 0u) atomicAdd(&P.counts[0], s_inst[g]);
+    if (!P.seq && inst_ok && tl0 == 0u && inst) atomicAdd(&P.counts[0], inst);
 #if PG_BANKCHK || PG_COALCHK
     __syncthreads();
     if (P.site_stats) {
