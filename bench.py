@@ -6,8 +6,8 @@ reduce0..reduce6 checked pairwise against reduce0 plus the injected off-by-one p
 per GPU (RAND32), checks EQUIV|RACE|OOB.  One step = every pair over the whole
 space: input generation (K1), both evaluation kernels (K2), comparison (K3),
 compaction (K4) and the H9 all_reduce of the first-counterexample key (MIN) and
-the counts (SUM).  Multi-GPU: every rank checks its own 64 seeds (seed_base =
-rank * 64), i.e. weak scaling; the only collective is H9.
+the counts (SUM).  Multi-GPU: N ranks shard a 64 x N seed space round-robin
+(64 seeds per GPU, weak scaling); the only collective is H9.
 
 `--impl reference` times the CPU oracle (oracle/, test infrastructure) on the
 host cores on a bounded sample of the same workload.
@@ -133,14 +133,15 @@ def _oracle_shard(args):
     return inst
 
 
-def oracle_sample(max_log_n=12, n_seeds=4):
+def oracle_sample(max_log_n=14, n_seeds=0):
     """The oracle as it stands, one process per host core over seed shards, on the
-    C2 pairs restricted to N <= 2^max_log_n and n_seeds seeds."""
+    C2 pairs restricted to N <= 2^max_log_n and n_seeds seeds (default: one seed per core)."""
     import multiprocessing as mp
     sys.path.insert(0, ROOT)
     import oracle
     oracle.build()
     cores = len(os.sched_getaffinity(0))
+    n_seeds = n_seeds or max(4, cores)
     world = min(cores, n_seeds)
     t0 = time.perf_counter()
     with mp.get_context("fork").Pool(world) as pool:
@@ -180,8 +181,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="pgvc", choices=["pgvc", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--ref-log-n", type=int, default=12)
-    ap.add_argument("--ref-seeds", type=int, default=4)
+    ap.add_argument("--ref-log-n", type=int, default=14)
+    ap.add_argument("--ref-seeds", type=int, default=0, help="0: one seed per host core")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + 1 step, no JSON (for ncu launch lists)")
     args = ap.parse_args()
     if args.impl == "reference":
@@ -194,7 +195,7 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    from paper_conf_ipps_lig12_b200 import build, pgvc
+    from paper_conf_ipps_lig12_b200 import build, distributed, pgvc
     if rank == 0 or world == 1:
         build.build()
     if world > 1:
@@ -220,14 +221,13 @@ def main():
             step_keys.fill_(2 ** 63 - 1)
             step_counts.zero_()
             for w in wls:
-                sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=w.n_seeds, seed_base=rank * SEEDS_PER_GPU,
+                # weak scaling: 64 seeds per GPU, seeds j = rank, rank + N, ... of a 64 x N seed space
+                sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=SEEDS_PER_GPU * world, rank=rank, world=world,
                                 checks=w.checks, stream=stream.cuda_stream, first_key=first_key, counts=counts)
                 runs.append(pgvc.check_equiv(irs[w.src], irs[w.tgt], sp))
                 torch.minimum(step_keys, first_key, out=step_keys)
                 step_counts.add_(counts)
-            if world > 1:   # H9: the only cross-GPU traffic
-                dist.all_reduce(step_keys, op=dist.ReduceOp.MIN)
-                dist.all_reduce(step_counts, op=dist.ReduceOp.SUM)
+            distributed.reduce_summary(step_keys, step_counts)   # H9: the only cross-GPU traffic
         return runs
 
     def collect(runs):

@@ -1,0 +1,72 @@
+"""Multi-process path on CPU (gloo, world_size 2): seed sharding + the H9 reduction
+(all_reduce MIN of first keys, SUM of counts) reproduce the single-process result.
+The oracle supplies per-shard results (no GPU here); the reduction code is the
+same `distributed.reduce_summary` bench.py runs over NCCL."""
+import os
+import socket
+
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, out):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    from paper_conf_ipps_lig12_b200 import distributed as D, workloads as W
+    w = W.c1(n_seeds=6)
+    ls = w.launch_src[::9]
+    r = oracle.check(W.subject(w.src), W.subject(w.tgt), ls, ls, n_seeds=6, rank=rank, world=world)
+    fk = torch.tensor(r["first_key"], dtype=torch.int64)
+    ct = torch.tensor(r["counts"], dtype=torch.int64)
+    D.reduce_summary(fk, ct)
+    out[rank] = (fk.tolist(), ct.tolist(), r["records"])
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.timeout(300)
+def test_gloo_world2_matches_single_process(oracle, W):
+    from paper_conf_ipps_lig12_b200 import distributed as D
+    mgr = mp.Manager()
+    out = mgr.dict()
+    port = _free_port()
+    mp.spawn(_worker, args=(2, port, out), nprocs=2, join=True)
+    w = W.c1(n_seeds=6)
+    ls = w.launch_src[::9]
+    full = oracle.check(W.subject(w.src), W.subject(w.tgt), ls, ls, n_seeds=6)
+    for rank in range(2):
+        fk, ct, _ = out[rank]
+        assert fk == full["first_key"]
+        # counts[11] (records) and [12] (failing instances) are per-rank sums too
+        assert ct == full["counts"]
+    merged = D.merge_records([out[0][2], out[1][2]])
+    assert merged == full["records"]
+    fw = D.first_witness(full["first_key"][0])
+    first_nonsquare = min(i for i, l in enumerate(ls) if l.bdim[0] != l.bdim[1])
+    assert fw["launch"] == first_nonsquare
+
+
+def test_fake_world_shards_union(oracle, W):
+    # sharding logic without any process group: shards r = 0..w-1 in one process
+    from paper_conf_ipps_lig12_b200 import distributed as D
+    w = W.c2_pair("reduce2", "reduce2_obo", n_seeds=5, max_log_n=6, max_log_b=4)
+    src, tgt = W.subject(w.src), W.subject(w.tgt)
+    full = oracle.check(src, tgt, w.launch_src, w.launch_tgt, n_seeds=5)
+    for world in (2, 3, 5):
+        parts = [oracle.check(src, tgt, w.launch_src, w.launch_tgt, n_seeds=5, rank=r, world=world)
+                 for r in range(world)]
+        assert D.merge_records([p["records"] for p in parts]) == full["records"]
+        assert min(p["first_key"][0] for p in parts) == full["first_key"][0]
+        assert [sum(p["counts"][i] for p in parts) for i in range(16)] == full["counts"]
