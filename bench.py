@@ -15,6 +15,7 @@ host cores on a bounded sample of the same workload.
 from __future__ import annotations
 
 import argparse
+import gc
 import json
 import os
 import statistics
@@ -184,6 +185,7 @@ def main():
     ap.add_argument("--ref-log-n", type=int, default=14)
     ap.add_argument("--ref-seeds", type=int, default=0, help="0: one seed per host core")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + 1 step, no JSON (for ncu launch lists)")
+    ap.add_argument("--diag", action="store_true", help="print per-step enqueue / device / per-check times")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)
@@ -214,78 +216,93 @@ def main():
     step_counts = torch.zeros(16, dtype=torch.int64, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 
-    def step():
-        """One pass of the whole path over the workload; returns (instances, runs)."""
+    def step(keys_out, counts_out):
+        """One pass of the whole path over the workload (enqueue only): H1..H8 per pair, H9 at the end."""
         runs = []
         with torch.cuda.stream(stream):
-            step_keys.fill_(2 ** 63 - 1)
-            step_counts.zero_()
+            keys_out.fill_(2 ** 63 - 1)
+            counts_out.zero_()
             for w in wls:
                 # weak scaling: 64 seeds per GPU, seeds j = rank, rank + N, ... of a 64 x N seed space
                 sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=SEEDS_PER_GPU * world, rank=rank, world=world,
                                 checks=w.checks, stream=stream.cuda_stream, first_key=first_key, counts=counts)
                 runs.append(pgvc.check_equiv(irs[w.src], irs[w.tgt], sp))
-                torch.minimum(step_keys, first_key, out=step_keys)
-                step_counts.add_(counts)
-            distributed.reduce_summary(step_keys, step_counts)   # H9: the only cross-GPU traffic
+                torch.minimum(keys_out, first_key, out=keys_out)
+                counts_out.add_(counts)
+            distributed.reduce_summary(keys_out, counts_out)   # H9: the only cross-GPU traffic
         return runs
 
     def collect(runs):
         d2h = 0
-        recs_total = 0
         for r in runs:
-            recs, s = r.collect(cap=1 << 16)
-            recs_total += len(recs)
+            recs, s = r.collect(cap=1 << 16, tuples=False)
             d2h += 64 * len(recs) + 8 * (16 + 11)
-        return d2h, recs_total
+        return d2h
 
-    # warm-up (also JIT-compiles every evaluation kernel variant)
+    # warm-up (also JIT-compiles every evaluation kernel variant and builds the plans)
     for _ in range(1 if args.profile else max(3, args.warmup)):
-        collect(step())
+        collect(step(step_keys, step_counts))
     torch.cuda.synchronize()
     if args.profile:
         torch.cuda.cudart().cudaProfilerStart()
-        collect(step())
+        collect(step(step_keys, step_counts))
         torch.cuda.synchronize()
         torch.cuda.cudart().cudaProfilerStop()
         return
 
+    # ---- device-timed phase: K steps enqueued back to back (L2 flush between steps, outside the
+    # timed events); host hiccups are absorbed by the queued work
+    keys = [torch.empty(11, dtype=torch.int64, device="cuda") for _ in range(args.steps)]
+    cnts = [torch.empty(16, dtype=torch.int64, device="cuda") for _ in range(args.steps)]
     clocks = Clocks(local)
+    gc.disable()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     clocks.start()
-    dev_ms, wall_s, inst_local, launches, h2d, d2h, eval_ms, n_k2, k2_inst = 0.0, 0.0, 0, 0, 0, 0, 0.0, 0, 0
-    for _ in range(args.steps):
-        flush.fill_(1)                       # L2 flush between timed steps (not timed)
-        torch.cuda.synchronize()
+    evs, all_runs = [], []
+    for k in range(args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(1)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        t0 = time.perf_counter()
         e0.record(stream)
-        runs = step()
+        all_runs.append(step(keys[k], cnts[k]))
         e1.record(stream)
-        dd, _ = collect(runs)                # records D2H (end-to-end result read)
-        wall_s += time.perf_counter() - t0
-        stream.synchronize()
-        dev_ms += e0.elapsed_time(e1)
-        d2h += dd
+        evs.append((e0, e1))
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    gc.enable()
+    step_ms = [e0.elapsed_time(e1) for e0, e1 in evs]
+    dev_ms = sum(step_ms)
+    inst_total = sum(int(c[0].item()) for c in cnts)      # whole job: counts are all-reduced over ranks
+    launches, h2d, eval_ms = 0, 0, 0.0
+    for runs in all_runs:
         for r in runs:
             t = r.timing()
             launches += t["launches"]
             h2d += t["h2d_bytes"]
             eval_ms += t["ms_eval"]
-        inst_local += int(step_counts[0].item()) if world == 1 else 0
-        if world > 1:
-            inst_local += int(step_counts[0].item())   # already all-reduced: whole-job instances
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    clk = clocks.stop()
+    if args.diag and rank == 0:
+        print("device ms per step:", ["%.1f" % x for x in step_ms], file=sys.stderr)
+    del all_runs
+
+    # ---- end-to-end phase: the same steps through the C ABI, host launch lists in, records and
+    # counters read back every step (wall clock)
+    wall_s, d2h = 0.0, 0
+    for k in range(args.steps):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        runs = step(keys[k], cnts[k])
+        d2h += collect(runs)
+        torch.cuda.synchronize()
+        wall_s += time.perf_counter() - t0
+        del runs
     t = torch.tensor([dev_ms, wall_s], dtype=torch.float64, device="cuda")
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     dev_ms, wall_s = float(t[0]), float(t[1])
-    inst_total = inst_local  # whole job (all ranks) per the all-reduced counts
     value = inst_total / (dev_ms / 1000.0)
     e2e = inst_total / wall_s
     peaks = measured_peaks()

@@ -464,7 +464,9 @@ struct Gen {
         o << "      default: return PG_END;\n    }\n";
         o << "R0:;\n" << body.str();
         o << "  }\n};\n\n";
-        o << "extern \"C\" __global__ void __launch_bounds__(1024, 1) pgk_eval(const PgParams P) { pg_main<PgK>(P); }\n";
+        o << "#ifndef PG_CTA_MAX\n#define PG_CTA_MAX 1024\n#define PG_MIN_BLOCKS 1\n#endif\n";
+        o << "extern \"C\" __global__ void __launch_bounds__(PG_CTA_MAX, PG_MIN_BLOCKS) pgk_eval(const PgParams P) "
+             "{ pg_main<PgK>(P); }\n";
         return o.str();
     }
 };

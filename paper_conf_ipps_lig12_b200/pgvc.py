@@ -47,6 +47,14 @@ class PgCex(ctypes.Structure):
         (n, ctypes.c_uint32) for n in REC_FIELDS[2:]]
 
 
+def _rec_dtype():
+    import numpy as np
+    return np.dtype([("key", "<u8"), ("count", "<u8")] + [(n, "<u4") for n in REC_FIELDS[2:]])
+
+
+REC_DTYPE = _rec_dtype()
+
+
 class PgSummary(ctypes.Structure):
     _fields_ = [("instances", ctypes.c_uint64), ("n_fail", ctypes.c_uint64), ("n_records", ctypes.c_uint64),
                 ("first_key", ctypes.c_int64), ("first_launch", ctypes.c_uint32),
@@ -203,13 +211,17 @@ class Run:
         self.space = space
         self._keep = keep
 
-    def collect(self, cap: int = 1 << 20):
+    def collect(self, cap: int = 1 << 20, tuples: bool = True):
+        """Synchronise, copy up to `cap` records.  Returns (records, summary): records as a
+        list of tuples in REC_FIELDS order (tuples=True) or a numpy structured array."""
+        import numpy as np
         n = ctypes.c_size_t()
         summ = PgSummary()
-        buf = (PgCex * max(1, cap))()
-        _ck(lib().pg_collect_cex(self._h, buf, cap, ctypes.byref(n), ctypes.byref(summ)))
-        m = min(n.value, cap)
-        recs = [tuple(getattr(buf[i], f) for f in REC_FIELDS) for i in range(m)]
+        buf = np.empty(max(1, cap), dtype=REC_DTYPE)
+        _ck(lib().pg_collect_cex(self._h, buf.ctypes.data_as(ctypes.POINTER(PgCex)), cap, ctypes.byref(n),
+                                 ctypes.byref(summ)))
+        arr = buf[:min(n.value, cap)]
+        recs = arr.tolist() if tuples else arr
         s = {"instances": summ.instances, "n_fail": summ.n_fail, "n_records": summ.n_records,
              "first_key": summ.first_key, "first_launch": summ.first_launch,
              "first_seed_idx": summ.first_seed_idx, "per_kind": list(summ.per_kind),
