@@ -112,7 +112,7 @@ def measured_peaks():
 
 def ncu_traffic():
     """Per-launch DRAM bytes of the evaluation kernel from the committed ncu capture (or None)."""
-    p = os.path.join(ROOT, "profiles", "k2_traffic.json")
+    p = os.path.join(ROOT, "profiles", "r1", "k2_traffic.json")
     try:
         with open(p) as f:
             return json.load(f).get("bytes_per_launch")

@@ -1,0 +1,17 @@
+#!/bin/bash
+# Run on the GPU box (gpurun): ncu evidence for one bench step of the headline workload.
+#   1. every launch of one step with its device time (cold-cache, serialised: compare shares)
+#   2. DRAM bytes and time of every evaluation-kernel launch (roofline "traffic")
+#   3. one `--set full` capture of the top evaluation-kernel launch (source-level, -lineinfo)
+set -u
+OUT=${1:-gpurun_out/prof}
+mkdir -p "$OUT/src"
+ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start off --csv \
+    --log-file "$OUT/launches.csv" python bench.py --profile > "$OUT/launches.log" 2>&1
+ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__warps_active.avg.pct_of_peak_sustained_active,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active \
+    --clock-control none --profile-from-start off -k regex:pgk_eval --csv \
+    --log-file "$OUT/k2_metrics.csv" python bench.py --profile > "$OUT/k2_metrics.log" 2>&1
+SKIP=${K2_SKIP:-2}
+PGVC_DUMP_SRC="$PWD/$OUT/src" ncu --set full --clock-control none --import-source on --profile-from-start off \
+    -k regex:pgk_eval -s "$SKIP" -c 1 -o "$OUT/k2_top" python bench.py --profile > "$OUT/k2_top.log" 2>&1
+echo done
