@@ -37,14 +37,33 @@ SM_COUNT = 148
 ALU_LANES_PER_SM_CLK = 64   # IADD3/LOP3 alu pipe: 4 SMSP x 16 lanes/clk (B300_MICROARCH: rt_SMSP = 2)
 
 
+WORKLOADS = {
+    # name: (description, seeds per GPU, ops per instance, builder(seeds))
+    "c2": ("C2: SDK reduce0 vs reduce1..6 + reduce2 vs reduce2_obo, B=2^0..2^10, N=B..2^16, "
+           "%d RAND32 seeds per GPU, checks EQUIV|RACE|OOB", 64, 13, lambda W, s: W.c2(n_seeds=s)),
+    "c1": ("C1: naive vs shared-memory transpose, bdim in [1,4]^2, up to 16x16 threads (1089 launches), "
+           "%d RAND32 seeds per GPU, checks EQUIV|RACE|OOB", 64, 14, lambda W, s: [W.c1(n_seeds=s)]),
+    "c3": ("C3: Blelloch scan vs padded scan (LOG_NUM_BANKS 4 and 5) and the dropped-barrier mutant, n <= 2^14, "
+           "%d seeds per GPU, checks EQUIV|RACE|OOB|BANK|COALESCE", 64, 15,
+           lambda W, s: [W.c3_pair("prescan_padded", 4, s), W.c3_pair("prescan_padded", 5, s),
+                         W.c3_pair("prescan_nobarrier", 4, s)]),
+    "c4": ("C4: bitonic global vs shared, n = 2^1..2^12, RAND32 + RANGE(4) x %d seeds per GPU + exhaustive 0/1 for "
+           "n <= 16", 64, 11, lambda W, s: W.c4("rand", s) + W.c4("range", s) + W.c4("bits")),
+    "c5t": ("C5 transpose: naive vs 32x32 tiled transpose, N = 32..1024, %d seeds per GPU", 1250, 14,
+            lambda W, s: [W.c5_transpose(n_seeds=s)]),
+    "c5m": ("C5 matmul: naive vs 32x32 tiled, N = 32..1024, K = 64, %d seeds per GPU", 1250, 10 * 64 + 10,
+            lambda W, s: [W.c5_matmul(n_seeds=s)]),
+}
+WL = "c2"
+
+
 def workload_desc():
-    return ("C2: SDK reduce0 vs reduce1..6 + reduce2 vs reduce2_obo, B=2^0..2^10, N=B..2^16, "
-            "%d RAND32 seeds per GPU, checks EQUIV|RACE|OOB" % SEEDS_PER_GPU)
+    return WORKLOADS[WL][0] % SEEDS_PER_GPU
 
 
 def c2_pairs():
     from paper_conf_ipps_lig12_b200 import workloads as W
-    return W.c2(n_seeds=SEEDS_PER_GPU)
+    return WORKLOADS[WL][3](W, SEEDS_PER_GPU)
 
 
 class Clocks:
@@ -186,7 +205,14 @@ def main():
     ap.add_argument("--ref-seeds", type=int, default=0, help="0: one seed per host core")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + 1 step, no JSON (for ncu launch lists)")
     ap.add_argument("--diag", action="store_true", help="print per-step enqueue / device / per-check times")
+    ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS),
+                    help="c2 (headline, BASELINE configs[1]); others: the remaining configs for reference")
+    ap.add_argument("--seeds", type=int, default=0, help="seeds per GPU (default: the workload's)")
     args = ap.parse_args()
+    global WL, SEEDS_PER_GPU, OPS_PER_INSTANCE
+    WL = args.workload
+    SEEDS_PER_GPU = args.seeds or WORKLOADS[WL][1]
+    OPS_PER_INSTANCE = WORKLOADS[WL][2]
     if args.impl == "reference":
         run_reference(args)
         return
@@ -224,7 +250,9 @@ def main():
             counts_out.zero_()
             for w in wls:
                 # weak scaling: 64 seeds per GPU, seeds j = rank, rank + N, ... of a 64 x N seed space
-                sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=SEEDS_PER_GPU * world, rank=rank, world=world,
+                ns = SEEDS_PER_GPU * world if w.input_mode != 1 else w.n_seeds   # exhaustive 0/1 sets are fixed
+                sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=ns, rank=rank, world=world,
+                                input_mode=w.input_mode, input_range=w.input_range,
                                 checks=w.checks, stream=stream.cuda_stream, first_key=first_key, counts=counts)
                 runs.append(pgvc.check_equiv(irs[w.src], irs[w.tgt], sp))
                 torch.minimum(keys_out, first_key, out=keys_out)
@@ -239,9 +267,16 @@ def main():
             d2h += 64 * len(recs) + 8 * (16 + 11)
         return d2h
 
-    # warm-up (also JIT-compiles every evaluation kernel variant and builds the plans)
-    for _ in range(1 if args.profile else max(3, args.warmup)):
-        collect(step(step_keys, step_counts))
+    # warm-up (also JIT-compiles every evaluation kernel variant, builds the plans, and sizes the
+    # memory pool for K steps in flight, the pattern of the device-timed phase)
+    collect(step(step_keys, step_counts))
+    if not args.profile:
+        for _ in range(max(1, args.warmup - 1)):
+            pending = [step(step_keys, step_counts) for _ in range(args.steps)]
+            torch.cuda.synchronize()
+            for runs in pending:
+                collect(runs)
+            del pending
     torch.cuda.synchronize()
     if args.profile:
         torch.cuda.cudart().cudaProfilerStart()

@@ -97,6 +97,7 @@ struct PgCold {     // per-emulated-thread state that lives in local memory
     u16 lsite[PG_WMAX];
     u32 ecnt[PG_NK];      // events per kind
     u32 ebest[PG_NK][8];  // minimum event per kind (X16)
+    u32 any;              // some event recorded
 };
 
 __device__ __forceinline__ bool pg_lex_less(const u32* a, const u32* b) {
@@ -115,6 +116,7 @@ __device__ __noinline__ void pg_event(PgCold& c, u32 kind, u32 round, u32 arr, u
         for (int i = 0; i < 8; i++) c.ebest[kind][i] = e[i];
     }
     c.ecnt[kind]++;
+    c.any = 1u;
 }
 
 // stamps: step (20 bits, >= 1) and block-local tid (12 bits)
@@ -418,6 +420,11 @@ __device__ __noinline__ void pg_race_check(u32 round, u32 step, u32 tlin, u32 gt
 
 template <int A, bool RD>
 __device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
+    if (pg_sL.T == 1u) {
+        pg_sh(t, PG_ARR(A).s_own)[flat] = pg_stamp_min(C, t);
+        pg_sh(t, PG_ARR(A).s_val)[flat] = val;
+        return;
+    }
     const u32 own = pg_sh(t, PG_ARR(A).s_own)[flat];
     if (own == pg_stamp_min(C, t)) pg_sh(t, PG_ARR(A).s_val)[flat] = val;
 #if PG_RACECHK
@@ -434,6 +441,12 @@ __device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& 
 
 template <int A, bool RD>
 __device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
+    if (pg_sL.T == 1u) {
+        t.arena[PG_ARR(A).off_own + flat] = pg_stamp_min(C, t);
+        t.arena[PG_ARR(A).off_val + flat] = val;
+        t.arena[PG_ARR(A).off_lw + flat] = t.gtid + 1u;
+        return;
+    }
     const u32 own = t.arena[PG_ARR(A).off_own + flat];
     if (own == pg_stamp_min(C, t)) {
         t.arena[PG_ARR(A).off_val + flat] = val;
@@ -453,7 +466,9 @@ __device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& 
 
 template <class K>
 __device__ __forceinline__ void pg_claim_all(const PgC& C, const PgT& t, const PgCold& c) {
-    if (t.nlog == 0u) return;
+    // a 1-thread block is the only writer of its cells in the round (other blocks sharing a
+    // global cell are an XB race and re-run sequentially): the check commits directly
+    if (t.nlog == 0u || pg_sL.T == 1u) return;
     K::claim_one(C, t, t.l0cell);
     for (u32 i = 1; i < t.nlog; i++) K::claim_one(C, t, c.lcell[i]);
 }
@@ -470,6 +485,7 @@ __device__ __forceinline__ void pg_check_all(const PgC& C, const PgT& t, PgCold&
 // successive warp-wide minima, counts by warp sum) and one lane updates the
 // (instance, kernel, kind) slot under its lock.  All 32 lanes call this.
 __device__ __noinline__ void pg_flush_warp(const PgParams& P, u32 lane, PgCold& c, u32 valid, u64 slot0) {
+    if (!__any_sync(PG_FULL, valid && c.any)) return;
     for (u32 k = 0; k < PG_NK; k++) {
         u32 pending = valid && c.ecnt[k] != 0u;
         for (;;) {
@@ -647,8 +663,11 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         t.sg = gc * gbytes;
         t.l0cell = t.l0val = t.l0site = 0u;
         for (u32 k = 0; k < PG_NK; k++) Cd[v].ecnt[k] = 0;
+        Cd[v].any = 0u;
         t.live = ok;
     }
+    __shared__ unsigned long long s_inst;
+    if (threadIdx.x == 0) s_inst = 0ull;
     __syncthreads();
     const bool grid_1d = pg_sL.gdim[1] == 1u && pg_sL.gdim[2] == 1u;
     u64 inst = 0;  // instances of this group (accumulated by its lane tl0 == 0)
@@ -753,7 +772,12 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         if (v >= V) break;
         pg_flush_warp(P, lane, Cd[v], inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)ms * pg_sW.slot_step);
     }
-    if (!P.seq && inst_ok && tl0 == 0u && inst) atomicAdd(&P.counts[0], inst);
+    // instances (X19): one shared atomic per group, one global atomic per CTA
+    if (!P.seq) {
+        if (inst_ok && tl0 == 0u && inst) atomicAdd(&s_inst, (unsigned long long)inst);
+        __syncthreads();
+        if (threadIdx.x == 0 && s_inst) atomicAdd(&P.counts[0], (u64)s_inst);
+    }
 #if PG_BANKCHK || PG_COALCHK
     __syncthreads();
     if (P.site_stats) {
