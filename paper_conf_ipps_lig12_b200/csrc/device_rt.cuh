@@ -480,49 +480,101 @@ __device__ __forceinline__ void pg_check_all(const PgC& C, const PgT& t, PgCold&
 }
 
 // ------------------------------------------------------------------ records (H8)
-// Each thread keeps its minimum event per kind; at the end of the CTA the lanes
-// of a warp that belong to the same instance merge theirs (lexicographic min by
-// successive warp-wide minima, counts by warp sum) and one lane updates the
-// (instance, kernel, kind) slot under its lock.  All 32 lanes call this.
-__device__ __noinline__ void pg_flush_warp(const PgParams& P, u32 lane, PgCold& c, u32 valid, u64 slot0) {
-    if (!__any_sync(PG_FULL, valid && c.any)) return;
+// Each thread keeps its minimum event per kind.  At the end of the CTA: (1) the
+// lanes of a warp that belong to the same instance merge (lexicographic min by
+// successive warp-wide minima, counts by warp sum); (2) warp leaders deposit
+// their results in shared memory and warp 0 merges entries of the same slot;
+// (3) one lane per (instance, kind) updates the global slot under its lock.
+// All threads of the CTA call pg_flush_cta.
+struct PgFlushEntry {
+    u64 slot;       // ~0: empty
+    u32 cnt;
+    u32 f[8];
+};
+
+__device__ __forceinline__ void pg_warp_merge(u32 pending, u64 key, u32 cnt_in, const u32* f_in, u32 lane,
+                                              u32& leader_out, u64& key_out, u32& cnt_out, u32* best, u32& members) {
+    const u32 pm = __ballot_sync(PG_FULL, pending);
+    const u32 leader = (u32)__ffs(pm) - 1u;
+    const u64 lkey = __shfl_sync(PG_FULL, key, leader);
+    u32 cand = pending && key == lkey;
+    members = __ballot_sync(PG_FULL, cand);
+    cnt_out = __reduce_add_sync(PG_FULL, cand ? cnt_in : 0u);
+#pragma unroll
+    for (int f = 0; f < 8; f++) {
+        best[f] = __reduce_min_sync(PG_FULL, cand ? f_in[f] : PG_NEVER);
+        cand = cand && f_in[f] == best[f];
+    }
+    leader_out = leader;
+    key_out = lkey;
+}
+
+__device__ __noinline__ void pg_slot_update(PgSlot* s, u32 cnt, const u32* best) {
+    atomicAdd(&s->count, (u64)cnt);
+    while (atomicCAS(&s->lock, 0u, 1u) != 0u) {
+    }
+    __threadfence();
+    volatile PgSlot* vs = s;
+    u32 cur[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) cur[i] = vs->f[i];
+    if (!vs->has || pg_lex_less(best, cur)) {
+#pragma unroll
+        for (int i = 0; i < 8; i++) vs->f[i] = best[i];
+        vs->has = 1u;
+    }
+    __threadfence();
+    atomicExch(&s->lock, 0u);
+}
+
+__device__ __noinline__ void pg_flush_cta(const PgParams& P, u32 lane, u32 warp, PgCold& c, u32 valid, u64 slot0,
+                                          PgFlushEntry* sh /* [32] in shared memory */) {
+    const u32 nwarps = blockDim.x >> 5;
     for (u32 k = 0; k < PG_NK; k++) {
+        if (!__syncthreads_or((int)(valid && c.ecnt[k] != 0u))) continue;
+        if (lane == 0) sh[warp].slot = ~0ull;
+        __syncwarp();
         u32 pending = valid && c.ecnt[k] != 0u;
+        bool first = true;
         for (;;) {
-            const u32 pm = __ballot_sync(PG_FULL, pending);
-            if (!pm) break;
-            const u32 leader = (u32)__ffs(pm) - 1u;
-            const u64 lslot = __shfl_sync(PG_FULL, slot0, leader);
-            u32 cand = pending && slot0 == lslot;
-            const u32 members = __ballot_sync(PG_FULL, cand);
-            const u32 cnt = __reduce_add_sync(PG_FULL, cand ? c.ecnt[k] : 0u);
-            u32 best[8];
-#pragma unroll
-            for (int f = 0; f < 8; f++) {
-                best[f] = __reduce_min_sync(PG_FULL, cand ? c.ebest[k][f] : PG_NEVER);
-                cand = cand && c.ebest[k][f] == best[f];
-            }
+            if (!__any_sync(PG_FULL, pending)) break;
+            u32 leader, cnt, members, best[8];
+            u64 key;
+            pg_warp_merge(pending, slot0, c.ecnt[k], c.ebest[k], lane, leader, key, cnt, best, members);
             if (lane == leader) {
-                PgSlot* s = P.slots + lslot + k;
-                atomicAdd(&s->count, (u64)cnt);
-                while (atomicCAS(&s->lock, 0u, 1u) != 0u) {
-                }
-                __threadfence();
-                volatile PgSlot* vs = s;
-                u32 cur[8];
+                if (first) {   // the common case: one instance per warp -> deposit for the CTA merge
+                    sh[warp].slot = key;
+                    sh[warp].cnt = cnt;
 #pragma unroll
-                for (int i = 0; i < 8; i++) cur[i] = vs->f[i];
-                if (!vs->has || pg_lex_less(best, cur)) {
-#pragma unroll
-                    for (int i = 0; i < 8; i++) vs->f[i] = best[i];
-                    vs->has = 1u;
+                    for (int i = 0; i < 8; i++) sh[warp].f[i] = best[i];
+                } else {
+                    pg_slot_update(P.slots + key + k, cnt, best);
                 }
-                __threadfence();
-                atomicExch(&s->lock, 0u);
             }
+            first = false;
             if (members & (1u << lane)) pending = 0u;
             __syncwarp();
         }
+        __syncthreads();
+        if (warp == 0) {
+            const bool has = lane < nwarps && sh[lane].slot != ~0ull;
+            u32 pend = has;
+            const u64 skey = has ? sh[lane].slot : 0ull;
+            const u32 scnt = has ? sh[lane].cnt : 0u;
+            u32 sf[8];
+#pragma unroll
+            for (int i = 0; i < 8; i++) sf[i] = has ? sh[lane].f[i] : PG_NEVER;
+            for (;;) {
+                if (!__any_sync(PG_FULL, pend)) break;
+                u32 leader, cnt, members, best[8];
+                u64 key;
+                pg_warp_merge(pend, skey, scnt, sf, lane, leader, key, cnt, best, members);
+                if (lane == leader) pg_slot_update(P.slots + key + k, cnt, best);
+                if (members & (1u << lane)) pend = 0u;
+                __syncwarp();
+            }
+        }
+        __syncthreads();
     }
 }
 
@@ -767,10 +819,22 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         }
     }
 #endif
+    {
+        __shared__ PgFlushEntry s_flush[32];
+        u32 any_ev = 0;
 #pragma unroll
-    for (u32 v = 0; v < PG_VMAX; v++) {
-        if (v >= V) break;
-        pg_flush_warp(P, lane, Cd[v], inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)ms * pg_sW.slot_step);
+        for (u32 v = 0; v < PG_VMAX; v++) {
+            if (v >= V) break;
+            any_ev |= Cd[v].any;
+        }
+        if (__syncthreads_or((int)any_ev)) {
+#pragma unroll
+            for (u32 v = 0; v < PG_VMAX; v++) {
+                if (v >= V) break;
+                pg_flush_cta(P, lane, warp, Cd[v], inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)ms * pg_sW.slot_step,
+                             s_flush);
+            }
+        }
     }
     // instances (X19): one shared atomic per group, one global atomic per CTA
     if (!P.seq) {
