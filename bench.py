@@ -220,9 +220,14 @@ def main():
     import torch
     import torch.distributed as dist
     world, rank, local = dist_env()
-    torch.cuda.set_device(local)
+    dev = local % max(1, torch.cuda.device_count())   # ranks > #GPUs share devices (tests only)
+    torch.cuda.set_device(dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("PGVC_DIST_BACKEND", "nccl")   # gloo: several ranks on one GPU (tests)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group(backend)
     from paper_conf_ipps_lig12_b200 import build, distributed, pgvc
     if rank == 0 or world == 1:
         build.build()
@@ -289,7 +294,7 @@ def main():
     # timed events); host hiccups are absorbed by the queued work
     keys = [torch.empty(11, dtype=torch.int64, device="cuda") for _ in range(args.steps)]
     cnts = [torch.empty(16, dtype=torch.int64, device="cuda") for _ in range(args.steps)]
-    clocks = Clocks(local)
+    clocks = Clocks(dev)
     gc.disable()
     if world > 1:
         dist.barrier()
