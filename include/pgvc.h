@@ -48,7 +48,8 @@ enum {
 };
 
 enum { PG_IN_RAND32 = 0, PG_IN_BITS01 = 1, PG_IN_RANGE = 2 };                 /* X8 */
-enum { PG_CHK_EQUIV = 1, PG_CHK_RACE = 2, PG_CHK_OOB = 4, PG_CHK_BANK = 8, PG_CHK_COALESCE = 16 };
+enum { PG_CHK_EQUIV = 1, PG_CHK_RACE = 2, PG_CHK_OOB = 4, PG_CHK_BANK = 8, PG_CHK_COALESCE = 16,
+       PG_CHK_DATAFLOW = 32 /* record the writer of every read (H5); evaluates blocks in bid order */ };
 enum { PG_BANKS_32 = 0, PG_BANKS_16_HALFWARP = 1 };                             /* X9 */
 enum {                                                                          /* X17 */
     PG_CEX_BARRIER_DIV = 0, PG_CEX_OOB = 1, PG_CEX_RACE_WW = 2, PG_CEX_RACE_RW = 3, PG_CEX_RACE_XB = 4,
@@ -135,6 +136,14 @@ int pg_collect_cex(pg_run *r, pg_cex *buf, size_t cap, size_t *n_written, pg_sum
  * accesses, conflicted|uncoalesced, max degree|sectors, sum degree|sectors,
  * sum ideal, sum active lanes, 0]; sites >= max_sites are dropped. */
 int pg_collect_site_stats(pg_run *r, uint64_t *buf, uint32_t max_sites);
+
+/* Data-flow relation of a run checked with PG_CHK_DATAFLOW (H5; the bounded form
+ * of the fresh-writer instantiation of Fig. 2): one row per in-bounds
+ * shared/global read, 12 x uint32 = [launch, seed_idx, block, round, gtid, site,
+ * array, addr, src (0 initial, 1 committed write, 2 own write this round),
+ * w_block, w_round, w_gtid] (0xFFFFFFFF for initial), in no particular order.
+ * *n_rows receives the number of reads (rows beyond the capacity are dropped). */
+int pg_collect_dataflow(pg_run *r, uint32_t *rows, size_t cap_rows, size_t *n_rows);
 
 /* Introspection of a loaded kernel. */
 int pg_ir_info(const pg_ir *k, uint32_t *n_sites, uint32_t *n_globals, uint32_t *n_scalars);

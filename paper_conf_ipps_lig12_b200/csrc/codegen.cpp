@@ -137,7 +137,7 @@ struct Gen {
             std::string src;
             if (n->ref < 3) src = "t.tid[" + std::to_string(c) + "]";
             else if (n->ref < 6) src = "t.bid[" + std::to_string(c) + "]";
-            else if (n->ref < 9) src = "pg_sL.bdim[" + std::to_string(c) + "]";
+            else if (n->ref < 9) src = "PG_BDIM" + std::to_string(c);
             else src = "pg_sL.gdim[" + std::to_string(c) + "]";
             return "pg_m(" + src + ")";
         }
@@ -419,6 +419,7 @@ struct Gen {
         o << "#define PG_BANKCHK " << ((O.checks & 8) ? 1 : 0) << "\n";
         o << "#define PG_COALCHK " << ((O.checks & 16) ? 1 : 0) << "\n";
         o << "#define PG_BANK16 " << (O.bank_model == 1 ? 1 : 0) << "\n";
+        o << "#define PG_DATAFLOW " << ((O.checks & 32) ? 1 : 0) << "\n";
         o << "#define PG_WMAX " << O.wmax << "\n";
         o << "#define PG_NSTATS " << std::max<size_t>(1, K.sites.size()) << "\n";
         o << "#ifndef PG_VMAX\n#define PG_VMAX 1\n#endif\n";

@@ -68,6 +68,38 @@ __shared__ PgWork pg_sW;                                    // this CTA's work i
 
 #define PG_ARR(A) (pg_sL.arr[A])
 
+// Launch-shape constants.  A variant compiled for one block shape (api.cpp,
+// shape_prelude) defines PG_S_*, and PgSA<A> for the shared-array layout: block
+// size, shared offsets and CTA packing become immediates.  Otherwise they are read
+// from the CTA's launch descriptor.
+#ifdef PG_S_T
+#define PG_T ((u32)PG_S_T)
+#define PG_BDIM0 ((u32)PG_S_B0)
+#define PG_BDIM1 ((u32)PG_S_B1)
+#define PG_BDIM2 ((u32)PG_S_B2)
+#define PG_SH(A, f) ((u32)PgSA<A>::f)
+#define PG_GBYTES ((u32)PG_S_GBYTES)
+#define PG_ZOFF ((u32)PG_S_ZOFF)
+#define PG_NOFF ((u32)PG_S_NOFF)
+#define PG_GPW ((u32)PG_S_GPW)
+#define PG_WPG ((u32)PG_S_WPG)
+#define PG_PK ((u32)PG_S_P)
+#define PG_VV ((u32)PG_S_V)
+#else
+#define PG_T (pg_sL.T)
+#define PG_BDIM0 (pg_sL.bdim[0])
+#define PG_BDIM1 (pg_sL.bdim[1])
+#define PG_BDIM2 (pg_sL.bdim[2])
+#define PG_SH(A, f) (pg_sL.arr[A].f)
+#define PG_GBYTES (pg_sL.smem_group_bytes)
+#define PG_ZOFF (pg_sL.smem_zero_off)
+#define PG_NOFF (pg_sL.smem_never_off)
+#define PG_GPW (pg_sL.gpw)
+#define PG_WPG (pg_sL.wpg)
+#define PG_PK (pg_sL.P)
+#define PG_VV (pg_sL.V)
+#endif
+
 struct PgC {        // CTA-uniform state
     u32 round;      // round index within the block (record field)
     u32 step;       // round counter of this CTA, >= 1 (stamps)
@@ -233,6 +265,34 @@ __device__ __forceinline__ void pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell
     }
 }
 
+#if PG_DATAFLOW
+struct PgDf {
+    u32* rows;
+    u32* count;
+    u64 seed_base;
+    u32 cap;
+};
+__shared__ PgDf pg_sDf;  // data-flow recorder of this CTA
+__device__ __noinline__ void pg_df_row(const PgC& C, const PgT& t, u32 site, u32 rec, u32 flat, u32 src, u32 wb, u32 wr,
+                                       u32 wg) {
+    const u32 i = atomicAdd(pg_sDf.count, 1u);
+    if (i >= pg_sDf.cap) return;
+    u32* r = pg_sDf.rows + (u64)i * 12u;
+    r[0] = pg_sW.launch;
+    r[1] = (u32)(t.seed - pg_sDf.seed_base);
+    r[2] = t.blk; r[3] = C.round; r[4] = t.gtid; r[5] = site; r[6] = rec; r[7] = flat;
+    r[8] = src; r[9] = wb; r[10] = wr; r[11] = wg;
+}
+// writer of a committed global cell: last committer (gtid) and the round of its stamp
+__device__ __forceinline__ void pg_df_global(const PgC& C, const PgT& t, u32 site, u32 rec, u32 flat, u32 lw, u32 own,
+                                             u64 off_step0) {
+    if (!lw) { pg_df_row(C, t, site, rec, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER); return; }
+    const u32 wg = lw - 1u, wb = wg / PG_T;
+    const u32 s0 = wb == t.blk ? C.step0 : t.arena[off_step0 + wb];
+    pg_df_row(C, t, site, rec, flat, 1u, wb, pg_owner_step(own) - s0, wg);
+}
+#endif
+
 __device__ __forceinline__ u32 pg_poison_sh(const PgT& t, u32 rec, u32 flat) {
     return pg_m(pg_rand32(t.seed, 0x8000u + (rec - 0x100u), ((u64)t.blk << 20) + flat));
 }
@@ -242,7 +302,7 @@ __device__ __forceinline__ u32 pg_poison_sh(const PgT& t, u32 rec, u32 flat) {
 // LOG: a load of A may follow a store to A in the same round (own-write lookup).
 template <int A, bool RD, bool LOG>
 __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site) {
-    const u32 inb = flat < PG_ARR(A).size;
+    const u32 inb = flat < PG_SH(A, size);
 #if PG_BANKCHK
     pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
 #endif
@@ -255,27 +315,39 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
         return pv;
     }
 #if PG_RACECHK
-    if (RD && pg_sL.T > 1u) {
-        atomicMin(pg_sh(t, PG_ARR(A).s_rmin) + flat, pg_stamp_min(C, t));
-        atomicMax(pg_sh(t, PG_ARR(A).s_rmax) + flat, pg_stamp_max(C, t));
+    if (RD && PG_T > 1u) {
+        atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + flat, pg_stamp_min(C, t));
+        atomicMax(pg_sh(t, PG_SH(A, s_rmax)) + flat, pg_stamp_max(C, t));
     }
 #endif
     u32 v;
-    if (LOG && pg_log_find(t, c, ((u32)A << 24) | flat, v)) return v;
-    const u32 own = pg_sh(t, PG_ARR(A).s_own)[flat];
+    if (LOG && pg_log_find(t, c, ((u32)A << 24) | flat, v)) {
+#if PG_DATAFLOW
+        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 2u, t.blk, C.round, t.gtid);
+#endif
+        return v;
+    }
+    const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
     if (pg_owner_step(own) < C.step0) {  // never written in this block (X6)
         const u32 pv = pg_poison_sh(t, PG_ARR(A).rec_id, flat);
 #if PG_OOBCHK
         pg_event(c, PGK_UNINIT, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
 #endif
+#if PG_DATAFLOW
+        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER);
+#endif
         return pv;
     }
-    return pg_sh(t, PG_ARR(A).s_val)[flat];
+#if PG_DATAFLOW
+    pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 1u, t.blk, pg_owner_step(own) - C.step0,
+              t.blk * PG_T + (own & 0xFFFu));
+#endif
+    return pg_sh(t, PG_SH(A, s_val))[flat];
 }
 
 template <int A>
 __device__ __forceinline__ void pg_st_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 val, u32 site) {
-    const u32 inb = flat < PG_ARR(A).size;
+    const u32 inb = flat < PG_SH(A, size);
 #if PG_BANKCHK
     pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
 #endif
@@ -317,13 +389,22 @@ __device__ __forceinline__ u32 pg_ld_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
     }
     pg_xb_mark<A>(t, flat);
 #if PG_RACECHK
-    if (RD && pg_sL.T > 1u) {
+    if (RD && PG_T > 1u) {
         atomicMin(t.arena + PG_ARR(A).off_rmin + flat, pg_stamp_min(C, t));
         atomicMax(t.arena + PG_ARR(A).off_rmax + flat, pg_stamp_max(C, t));
     }
 #endif
     u32 v;
-    if (LOG && pg_log_find(t, c, ((u32)A << 24) | flat, v)) return v;
+    if (LOG && pg_log_find(t, c, ((u32)A << 24) | flat, v)) {
+#if PG_DATAFLOW
+        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 2u, t.blk, C.round, t.gtid);
+#endif
+        return v;
+    }
+#if PG_DATAFLOW
+    pg_df_global(C, t, site, PG_ARR(A).rec_id, flat, t.arena[PG_ARR(A).off_lw + flat],
+                 t.arena[PG_ARR(A).off_own + flat], pg_sL.off_step0);
+#endif
     return t.arena[PG_ARR(A).off_val + flat];
 }
 
@@ -359,6 +440,9 @@ __device__ __forceinline__ u32 pg_ld_gi(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
 #endif
         return pv;
     }
+#if PG_DATAFLOW
+    pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER);
+#endif
     return __ldg(t.input + PG_ARR(A).off_in + flat);
 }
 
@@ -388,16 +472,16 @@ __device__ __forceinline__ void pg_tick(PgC& C, PgT& t, PgCold& c, u32 act) {
 // the owner reports WW, and the thread the X16 rule names tid_a reports RW.
 template <int A>
 __device__ __forceinline__ void pg_claim_sh(const PgC& C, const PgT& t, u32 flat) {
-    atomicMin(pg_sh(t, PG_ARR(A).s_own) + flat, pg_stamp_min(C, t));
+    atomicMin(pg_sh(t, PG_SH(A, s_own)) + flat, pg_stamp_min(C, t));
 #if PG_RACECHK
-    if (pg_sL.T > 1u) atomicMax(pg_sh(t, PG_ARR(A).s_wmax) + flat, pg_stamp_max(C, t));
+    if (PG_T > 1u) atomicMax(pg_sh(t, PG_SH(A, s_wmax)) + flat, pg_stamp_max(C, t));
 #endif
 }
 template <int A>
 __device__ __forceinline__ void pg_claim_gt(const PgC& C, const PgT& t, u32 flat) {
     atomicMin(t.arena + PG_ARR(A).off_own + flat, pg_stamp_min(C, t));
 #if PG_RACECHK
-    if (pg_sL.T > 1u) atomicMax(t.arena + PG_ARR(A).off_wmax + flat, pg_stamp_max(C, t));
+    if (PG_T > 1u) atomicMax(t.arena + PG_ARR(A).off_wmax + flat, pg_stamp_max(C, t));
 #endif
 }
 
@@ -420,18 +504,18 @@ __device__ __noinline__ void pg_race_check(u32 round, u32 step, u32 tlin, u32 gt
 
 template <int A, bool RD>
 __device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
-    if (pg_sL.T == 1u) {
-        pg_sh(t, PG_ARR(A).s_own)[flat] = pg_stamp_min(C, t);
-        pg_sh(t, PG_ARR(A).s_val)[flat] = val;
+    if (PG_T == 1u) {
+        pg_sh(t, PG_SH(A, s_own))[flat] = pg_stamp_min(C, t);
+        pg_sh(t, PG_SH(A, s_val))[flat] = val;
         return;
     }
-    const u32 own = pg_sh(t, PG_ARR(A).s_own)[flat];
-    if (own == pg_stamp_min(C, t)) pg_sh(t, PG_ARR(A).s_val)[flat] = val;
+    const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
+    if (own == pg_stamp_min(C, t)) pg_sh(t, PG_SH(A, s_val))[flat] = val;
 #if PG_RACECHK
-    if (pg_sL.T > 1u) {
-        const u32 wmax = pg_sh(t, PG_ARR(A).s_wmax)[flat];
-        const u32 rmin = RD ? pg_sh(t, PG_ARR(A).s_rmin)[flat] : 0u;
-        const u32 rmax = RD ? pg_sh(t, PG_ARR(A).s_rmax)[flat] : 0u;
+    if (PG_T > 1u) {
+        const u32 wmax = pg_sh(t, PG_SH(A, s_wmax))[flat];
+        const u32 rmin = RD ? pg_sh(t, PG_SH(A, s_rmin))[flat] : 0u;
+        const u32 rmax = RD ? pg_sh(t, PG_SH(A, s_rmax))[flat] : 0u;
         if ((wmax & 0xFFFu) != (own & 0xFFFu) || (RD && (rmax >> 12) == C.step))
             pg_race_check(C.round, C.step, t.tlin, t.gtid, c, val, site, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin,
                           rmax);
@@ -441,7 +525,7 @@ __device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& 
 
 template <int A, bool RD>
 __device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
-    if (pg_sL.T == 1u) {
+    if (PG_T == 1u) {
         t.arena[PG_ARR(A).off_own + flat] = pg_stamp_min(C, t);
         t.arena[PG_ARR(A).off_val + flat] = val;
         t.arena[PG_ARR(A).off_lw + flat] = t.gtid + 1u;
@@ -453,7 +537,7 @@ __device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& 
         t.arena[PG_ARR(A).off_lw + flat] = t.gtid + 1u;
     }
 #if PG_RACECHK
-    if (pg_sL.T > 1u) {
+    if (PG_T > 1u) {
         const u32 wmax = t.arena[PG_ARR(A).off_wmax + flat];
         const u32 rmin = RD ? t.arena[PG_ARR(A).off_rmin + flat] : 0u;
         const u32 rmax = RD ? t.arena[PG_ARR(A).off_rmax + flat] : 0u;
@@ -468,7 +552,7 @@ template <class K>
 __device__ __forceinline__ void pg_claim_all(const PgC& C, const PgT& t, const PgCold& c) {
     // a 1-thread block is the only writer of its cells in the round (other blocks sharing a
     // global cell are an XB race and re-run sequentially): the check commits directly
-    if (t.nlog == 0u || pg_sL.T == 1u) return;
+    if (t.nlog == 0u || PG_T == 1u) return;
     K::claim_one(C, t, t.l0cell);
     for (u32 i = 1; i < t.nlog; i++) K::claim_one(C, t, c.lcell[i]);
 }
@@ -609,6 +693,9 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         u32* wd = (u32*)&pg_sW;
         for (u32 i = threadIdx.x; i < sizeof(PgWork) / 4; i += blockDim.x) wd[i] = ws[i];
     }
+#if PG_DATAFLOW
+    if (threadIdx.x == 0) pg_sDf = PgDf{P.df_rows, P.df_count, P.seed_base, P.df_cap};
+#endif
     __syncthreads();
     const u32 G = pg_sW.ngroups, GB = pg_sW.gb;
     if (P.seq) {
@@ -647,19 +734,19 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         __threadfence();
         __syncthreads();
     }
-    const u32 gbytes = pg_sL.smem_group_bytes;
-    const u32 T_ = pg_sL.T;
+    const u32 gbytes = PG_GBYTES;
+    const u32 T_ = PG_T;
     const bool warp_blocks = T_ <= 32u;  // an emulated block never spans warps: warp-level barriers suffice
-    u64* sstats = (u64*)(pg_dsmem + (u64)pg_sL.P * gbytes);
+    u64* sstats = (u64*)(pg_dsmem + (u64)PG_PK * gbytes);
     u32* s_grounds = (u32*)(sstats + ((PG_BANKCHK || PG_COALCHK) ? PG_NSTATS * 8 : 0));  // per group (T > 32)
     // shared regions: initialised once per CTA (stamps are step-tagged)
     {
-        const u32 zw = (pg_sL.smem_never_off - pg_sL.smem_zero_off) / 4u;
-        const u32 nw = (gbytes - pg_sL.smem_never_off) / 4u;
+        const u32 zw = (PG_NOFF - PG_ZOFF) / 4u;
+        const u32 nw = (gbytes - PG_NOFF) / 4u;
         const u32 per = zw + nw;
         for (u32 i = threadIdx.x; i < G * per; i += blockDim.x) {
             const u32 gi = i / per, j = i - gi * per;
-            u32* base = (u32*)(pg_dsmem + (u64)gi * gbytes + pg_sL.smem_zero_off);
+            u32* base = (u32*)(pg_dsmem + (u64)gi * gbytes + PG_ZOFF);
             base[j] = j < zw ? 0u : PG_NEVER;
         }
     }
@@ -668,7 +755,7 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
 #else
     sstats = nullptr;
 #endif
-    for (u32 i = threadIdx.x; i < pg_sL.P; i += blockDim.x) s_grounds[i] = 0;
+    for (u32 i = threadIdx.x; i < PG_PK; i += blockDim.x) s_grounds[i] = 0;
 
     PgC C;
     C.step = 0;
@@ -677,16 +764,16 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
     u32 g, tl0, lane_ok, ekey, gmask;
     if (warp_blocks) {
         const u32 sub = lane / T_;
-        g = warp * pg_sL.gpw + sub;
+        g = warp * PG_GPW + sub;
         tl0 = lane - sub * T_;
-        lane_ok = sub < pg_sL.gpw;
+        lane_ok = sub < PG_GPW;
         ekey = lane_ok ? sub : 63u;
-        const u32 span = pg_sL.gpw * T_;
+        const u32 span = PG_GPW * T_;
         gmask = lane_ok ? (T_ == 32u ? PG_FULL : (((1u << T_) - 1u) << (sub * T_)))
                         : (span >= 32u ? 0u : ~((1u << span) - 1u));
     } else {
-        g = warp / pg_sL.wpg;
-        tl0 = (warp % pg_sL.wpg) * 32u + lane;
+        g = warp / PG_WPG;
+        tl0 = (warp % PG_WPG) * 32u + lane;
         lane_ok = 1u;
         ekey = 0u;
         gmask = PG_FULL;
@@ -697,7 +784,7 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
     typename K::Frame F[PG_VMAX];
     PgT T[PG_VMAX];
     PgCold Cd[PG_VMAX];
-    const u32 V = PG_VMAX > 1 ? pg_sL.V : 1u;
+    const u32 V = PG_VMAX > 1 ? PG_VV : 1u;
 #pragma unroll
     for (u32 v = 0; v < PG_VMAX; v++) {
         if (v >= V) break;
@@ -706,9 +793,9 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         const u32 ok = inst_ok && t.tlin < T_;
         t.ekey = ok ? ekey : 63u;
         t.lane = lane;
-        t.tid[0] = t.tlin % pg_sL.bdim[0];
-        t.tid[1] = (t.tlin / pg_sL.bdim[0]) % pg_sL.bdim[1];
-        t.tid[2] = t.tlin / (pg_sL.bdim[0] * pg_sL.bdim[1]);
+        t.tid[0] = t.tlin % PG_BDIM0;
+        t.tid[1] = (t.tlin / PG_BDIM0) % PG_BDIM1;
+        t.tid[2] = t.tlin / (PG_BDIM0 * PG_BDIM1);
         t.seed = P.seed_base + (u64)(pg_sW.seed_j0 + ms * pg_sW.seed_jstep);
         t.arena = P.arena + pg_sW.arena_off + (u64)ms * pg_sL.arena_stride;
         t.input = P.input + pg_sW.input_off + (u64)ms * pg_sL.input_stride;
@@ -746,6 +833,9 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
             t.gtid = blk * T_ + t.tlin;
             K::init(F[v], C, t);
         }
+#if PG_DATAFLOW
+        if (pg_sL.off_step0 != ~0ull && inst_ok && tl0 == 0u && blk_ok) T[0].arena[pg_sL.off_step0 + blk] = C.step0;
+#endif
         C.round = 0;
         u32 resume = 0;
         for (;;) {
@@ -837,7 +927,7 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         }
     }
     // instances (X19): one shared atomic per group, one global atomic per CTA
-    if (!P.seq) {
+    if (P.count_inst) {
         if (inst_ok && tl0 == 0u && inst) atomicAdd(&s_inst, (unsigned long long)inst);
         __syncthreads();
         if (threadIdx.x == 0 && s_inst) atomicAdd(&P.counts[0], (u64)s_inst);

@@ -48,6 +48,7 @@ struct PgLaunchK {
     // per-group shared region: [values | stamps starting at 0 | stamps starting at ~0]
     u32 smem_group_bytes, smem_zero_off, smem_never_off, n_arrays;
     u64 arena_stride, input_stride;          // u32 words per instance
+    u64 off_step0;                           // data-flow mode: per-block first round step (arena words), ~0 absent
     PgArr arr[PG_MAXARR];
 };
 
@@ -88,7 +89,11 @@ struct PgParams {
     u32 fuel;
     u32 seq;           // 0: block-parallel pass; 1: sequential re-run of flagged seed groups
     u32 input_mode, input_range, mask;
-    u32 pad;
+    u32 count_inst;    // this pass counts instances (X19)
+    u32* df_rows;      // data-flow rows (12 words each), PG_CHK_DATAFLOW only
+    u32* df_count;
+    u32 df_cap;
+    u32 pad2;
 };
 
 // K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive

@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(_HERE, "libpgvc.so")
 
 PG_OK, PG_E_ARG, PG_E_PARSE, PG_E_TYPE, PG_E_LIMIT, PG_E_CUDA, PG_E_OOM, PG_E_STATE = 0, -1, -2, -3, -4, -5, -6, -7
 IN_RAND32, IN_BITS01, IN_RANGE = 0, 1, 2
-CHK_EQUIV, CHK_RACE, CHK_OOB, CHK_BANK, CHK_COALESCE = 1, 2, 4, 8, 16
+CHK_EQUIV, CHK_RACE, CHK_OOB, CHK_BANK, CHK_COALESCE, CHK_DATAFLOW = 1, 2, 4, 8, 16, 32
 BANKS_32, BANKS_16_HALFWARP = 0, 1
 KINDS = ["BARRIER_DIV", "OOB", "RACE_WW", "RACE_RW", "RACE_XB", "MISMATCH", "BANK", "UNCOALESCED", "UNINIT", "LIMIT"]
 N_KINDS = 10
@@ -38,6 +38,8 @@ class PgSpace(ctypes.Structure):
                 ("d_first_key", ctypes.c_void_p), ("d_counts", ctypes.c_void_p)]
 
 
+DF_FIELDS = ("launch", "seed_idx", "block", "round", "gtid", "site", "array", "addr", "src", "w_block",
+             "w_round", "w_gtid")
 REC_FIELDS = ("key", "count", "kind", "launch", "seed_idx", "kernel", "round", "site", "array", "addr",
               "tid_a", "tid_b", "val_a", "val_b")
 
@@ -70,7 +72,7 @@ class PgError(RuntimeError):
 
 _lib = None
 EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_collect_cex",
-           "pg_collect_site_stats", "pg_ir_info", "pg_ir_source", "pg_ir_compile", "pg_run_timing",
+           "pg_collect_site_stats", "pg_collect_dataflow", "pg_ir_info", "pg_ir_source", "pg_ir_compile", "pg_run_timing",
            "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
 
 
@@ -91,6 +93,8 @@ def lib():
     L.pg_collect_cex.argtypes = [vp, ctypes.POINTER(PgCex), ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t),
                                  ctypes.POINTER(PgSummary)]
     L.pg_collect_site_stats.argtypes = [vp, ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32]
+    L.pg_collect_dataflow.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.c_size_t,
+                                      ctypes.POINTER(ctypes.c_size_t)]
     L.pg_ir_info.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32),
                              ctypes.POINTER(ctypes.c_uint32)]
     L.pg_ir_source.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_char_p,
@@ -103,7 +107,8 @@ def lib():
     L.pg_ir_free.argtypes = [vp]
     L.pg_run_free.argtypes = [vp]
     for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_collect_cex",
-              "pg_collect_site_stats", "pg_ir_info", "pg_ir_source", "pg_ir_compile", "pg_run_timing"):
+              "pg_collect_site_stats", "pg_collect_dataflow", "pg_ir_info", "pg_ir_source", "pg_ir_compile",
+              "pg_run_timing"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -234,6 +239,18 @@ class Run:
         out = np.zeros((nl, 2, max_sites, 8), dtype=np.uint64)
         _ck(lib().pg_collect_site_stats(self._h, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), max_sites))
         return out
+
+    def dataflow(self):
+        """Data-flow rows of a run checked with CHK_DATAFLOW: uint32 array (n, 12) in
+        DF_FIELDS order, sorted lexicographically."""
+        import numpy as np
+        n = ctypes.c_size_t()
+        _ck(lib().pg_collect_dataflow(self._h, None, 0, ctypes.byref(n)))
+        out = np.zeros((max(1, n.value), 12), dtype=np.uint32)
+        _ck(lib().pg_collect_dataflow(self._h, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)), n.value,
+                                      ctypes.byref(n)))
+        out = out[:min(n.value, 1 << 20)]
+        return out[np.lexsort(out.T[::-1])] if len(out) else out
 
     def timing(self):
         a, b, n, h = ctypes.c_float(), ctypes.c_float(), ctypes.c_uint32(), ctypes.c_uint64()
