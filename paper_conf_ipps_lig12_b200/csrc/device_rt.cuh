@@ -32,8 +32,15 @@ __device__ __forceinline__ i32 pg_sx(u32 v) {
 __device__ __forceinline__ u32 pg_add(u32 a, u32 b) { return pg_m(a + b); }
 __device__ __forceinline__ u32 pg_sub(u32 a, u32 b) { return pg_m(a - b); }
 __device__ __forceinline__ u32 pg_mul(u32 a, u32 b) { return pg_m(a * b); }
-__device__ __forceinline__ u32 pg_udiv(u32 a, u32 b) { return b ? a / b : PG_MASK; }
-__device__ __forceinline__ u32 pg_urem(u32 a, u32 b) { return b ? a % b : a; }
+// power-of-two divisors (e.g. the SDK reductions' 2*s) take the shift/mask identity
+__device__ __forceinline__ u32 pg_udiv(u32 a, u32 b) {
+    if (b && !(b & (b - 1u))) return a >> (__ffs(b) - 1);
+    return b ? a / b : PG_MASK;
+}
+__device__ __forceinline__ u32 pg_urem(u32 a, u32 b) {
+    if (b && !(b & (b - 1u))) return a & (b - 1u);
+    return b ? a % b : a;
+}
 __device__ __forceinline__ u32 pg_sdiv(u32 a, u32 b) {
     i32 x = pg_sx(a), y = pg_sx(b);
     if (y == 0) return x < 0 ? 1u : PG_MASK;
@@ -516,7 +523,9 @@ __device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& 
         const u32 wmax = pg_sh(t, PG_SH(A, s_wmax))[flat];
         const u32 rmin = RD ? pg_sh(t, PG_SH(A, s_rmin))[flat] : 0u;
         const u32 rmax = RD ? pg_sh(t, PG_SH(A, s_rmax))[flat] : 0u;
-        if ((wmax & 0xFFFu) != (own & 0xFFFu) || (RD && (rmax >> 12) == C.step))
+        // (a cell only its writer read this round is no RW race: skip the slow path)
+        if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
+            (RD && (rmax >> 12) == C.step && (((rmin ^ own) | (rmax ^ own)) & 0xFFFu)))
             pg_race_check(C.round, C.step, t.tlin, t.gtid, c, val, site, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin,
                           rmax);
     }
@@ -541,7 +550,9 @@ __device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& 
         const u32 wmax = t.arena[PG_ARR(A).off_wmax + flat];
         const u32 rmin = RD ? t.arena[PG_ARR(A).off_rmin + flat] : 0u;
         const u32 rmax = RD ? t.arena[PG_ARR(A).off_rmax + flat] : 0u;
-        if ((wmax & 0xFFFu) != (own & 0xFFFu) || (RD && (rmax >> 12) == C.step))
+        // (a cell only its writer read this round is no RW race: skip the slow path)
+        if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
+            (RD && (rmax >> 12) == C.step && (((rmin ^ own) | (rmax ^ own)) & 0xFFFu)))
             pg_race_check(C.round, C.step, t.tlin, t.gtid, c, val, site, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin,
                           rmax);
     }
@@ -683,13 +694,13 @@ __device__ __forceinline__ u32 pg_init_value(const PgParams& P, u64 seed, u32 gi
 }
 
 template <class K>
-__device__ __forceinline__ void pg_main(const PgParams& P) {
+__device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     __shared__ u32 s_flag;
     {
-        const u32* src = (const u32*)&P.launches[P.work[blockIdx.x].launch];
+        const u32* src = (const u32*)&P.launches[P.work[wi].launch];
         u32* dst = (u32*)&pg_sL;
         for (u32 i = threadIdx.x; i < sizeof(PgLaunchK) / 4; i += blockDim.x) dst[i] = src[i];
-        const u32* ws = (const u32*)&P.work[blockIdx.x];
+        const u32* ws = (const u32*)&P.work[wi];
         u32* wd = (u32*)&pg_sW;
         for (u32 i = threadIdx.x; i < sizeof(PgWork) / 4; i += blockDim.x) wd[i] = ws[i];
     }
@@ -761,22 +772,18 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
     C.step = 0;
     C.fuel = P.fuel;
     const u32 lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-    u32 g, tl0, lane_ok, ekey, gmask;
+    u32 g, tl0, lane_ok, ekey;
     if (warp_blocks) {
         const u32 sub = lane / T_;
         g = warp * PG_GPW + sub;
         tl0 = lane - sub * T_;
         lane_ok = sub < PG_GPW;
         ekey = lane_ok ? sub : 63u;
-        const u32 span = PG_GPW * T_;
-        gmask = lane_ok ? (T_ == 32u ? PG_FULL : (((1u << T_) - 1u) << (sub * T_)))
-                        : (span >= 32u ? 0u : ~((1u << span) - 1u));
     } else {
         g = warp / PG_WPG;
         tl0 = (warp % PG_WPG) * 32u + lane;
         lane_ok = 1u;
         ekey = 0u;
-        gmask = PG_FULL;
     }
     const u32 inst_ok = lane_ok && g < G;
     const u32 gc = inst_ok ? g : 0u;
@@ -805,8 +812,7 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         Cd[v].any = 0u;
         t.live = ok;
     }
-    __shared__ unsigned long long s_inst;
-    if (threadIdx.x == 0) s_inst = 0ull;
+    __shared__ u64 s_part[32];   // per-warp instance counts
     __syncthreads();
     const bool grid_1d = pg_sL.gdim[1] == 1u && pg_sL.gdim[2] == 1u;
     u64 inst = 0;  // instances of this group (accumulated by its lane tl0 == 0)
@@ -873,9 +879,18 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         }
         // rounds of this group's block = max over its threads of the rounds they entered alive
         u32 grounds;
-        if (warp_blocks) {
-            grounds = __reduce_max_sync(PG_FULL, 0u);  // keep the warp converged before the segmented max
-            grounds = gmask ? __reduce_max_sync(gmask, alive_rounds) : 0u;
+        if (warp_blocks && (T_ & (T_ - 1u)) == 0u) {
+            // groups are aligned power-of-two lane segments: butterfly max (no per-group masks,
+            // which would serialise the warp once per group)
+            grounds = alive_rounds;
+            for (u32 o = 1u; o < T_; o <<= 1) grounds = max(grounds, __shfl_xor_sync(PG_FULL, grounds, o));
+        } else if (warp_blocks) {
+            if (inst_ok && alive_rounds) atomicMax(&s_grounds[g], alive_rounds);
+            __syncwarp();
+            grounds = inst_ok ? s_grounds[g] : 0u;
+            __syncwarp();
+            if (inst_ok && tl0 == 0u) s_grounds[g] = 0u;
+            __syncwarp();
         } else {
             if (inst_ok && alive_rounds) atomicMax(&s_grounds[g], alive_rounds);
             __syncthreads();
@@ -926,11 +941,18 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
             }
         }
     }
-    // instances (X19): one shared atomic per group, one global atomic per CTA
+    // instances (X19): warp sums, then one global atomic per CTA
     if (P.count_inst) {
-        if (inst_ok && tl0 == 0u && inst) atomicAdd(&s_inst, (unsigned long long)inst);
+        u64 x = (inst_ok && tl0 == 0u) ? inst : 0ull;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(PG_FULL, x, o);
+        if (lane == 0u) s_part[warp] = x;
         __syncthreads();
-        if (threadIdx.x == 0 && s_inst) atomicAdd(&P.counts[0], (u64)s_inst);
+        if (threadIdx.x == 0) {
+            u64 sum = 0;
+            for (u32 w = 0; w < (blockDim.x + 31u) / 32u; w++) sum += s_part[w];
+            if (sum) atomicAdd(&P.counts[0], sum);
+        }
     }
 #if PG_BANKCHK || PG_COALCHK
     __syncthreads();
@@ -944,4 +966,16 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
         }
     }
 #endif
+}
+
+// One work item per CTA, or (sequential pass) a grid-stride loop over the items the
+// selection kernel listed: a pass with nothing to re-run costs one short launch.
+template <class K>
+__device__ __forceinline__ void pg_main(const PgParams& P) {
+    const bool listed = P.work_count != nullptr;
+    const u32 n = listed ? *P.work_count : blockIdx.x + 1u;
+    for (u32 i = blockIdx.x; i < n; i += gridDim.x) {   // (one call site: one inlined copy)
+        pg_item<K>(P, listed ? P.work_list[i] : i);
+        __syncthreads();
+    }
 }

@@ -108,6 +108,17 @@ __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ job
     }
 }
 
+// K2b': list the sequential-pass items whose seed group has a flagged instance.
+__global__ void __launch_bounds__(256) pg_seq_select(const PgWork* __restrict__ items, u32 n_items,
+                                                     const u32* flags, u32* list, u32* count) {
+    const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n_items) return;
+    const PgWork w = items[i];
+    u32 f = 0;
+    for (u32 s = 0; s < w.nseeds; s++) f |= flags[w.inst0 + s];
+    if (f) list[atomicAdd(count, 1u)] = i;
+}
+
 // K2c: fold the per-item site statistics of the block-parallel pass into the
 // per-launch table, skipping seed groups that the sequential pass re-runs.
 __global__ void __launch_bounds__(128) pg_stats_reduce(const PgWork* __restrict__ items, const u64* item_stats,
@@ -281,6 +292,12 @@ cudaError_t xb_detect(const PgXb* jobs, u32 n_jobs, u32 max_inst, const u32* are
         dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
         pg_xb_detect<<<grid, 256, 0, st>>>(jobs + j0, arena, flags);
     }
+    return cudaGetLastError();
+}
+
+cudaError_t seq_select(const PgWork* items, u32 n_items, const u32* flags, u32* list, u32* count, cudaStream_t st) {
+    if (!n_items) return cudaSuccess;
+    pg_seq_select<<<(n_items + 255) / 256, 256, 0, st>>>(items, n_items, flags, list, count);
     return cudaGetLastError();
 }
 

@@ -94,6 +94,8 @@ struct PgParams {
     u32* df_count;
     u32 df_cap;
     u32 pad2;
+    const u32* work_list;   // sequential pass: indices (into work) of the items to run
+    const u32* work_count;  // their number (device); nullptr: one item per CTA
 };
 
 // K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive

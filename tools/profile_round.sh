@@ -11,7 +11,22 @@ ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start o
 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__warps_active.avg.pct_of_peak_sustained_active,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active \
     --clock-control none --profile-from-start off -k regex:pgk_eval --csv \
     --log-file "$OUT/k2_metrics.csv" python bench.py --profile > "$OUT/k2_metrics.log" 2>&1
-SKIP=${K2_SKIP:-2}
+# the longest evaluation-kernel launch of the metrics pass (same filter => same launch index)
+SKIP=${K2_SKIP:-$(python - "$OUT/k2_metrics.csv" <<'PY'
+import csv, sys
+best, idx, seen = -1.0, 0, {}
+for r in csv.reader(open(sys.argv[1])):
+    if len(r) > 14 and r[0].isdigit() and r[12] == "gpu__time_duration.sum":
+        i = int(r[0])
+        if i not in seen:
+            seen[i] = len(seen)
+        v = float(r[14].replace(",", ""))
+        if v > best:
+            best, idx = v, seen[i]
+print(idx)
+PY
+)}
+echo "k2 top launch index: $SKIP"
 PGVC_DUMP_SRC="$PWD/$OUT/src" ncu --set full --clock-control none --import-source on --profile-from-start off \
     -k regex:pgk_eval -s "$SKIP" -c 1 -o "$OUT/k2_top" python bench.py --profile > "$OUT/k2_top.log" 2>&1
 echo done
