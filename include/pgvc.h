@@ -126,6 +126,17 @@ int pg_check_races(const pg_ir *k, const pg_space *sp, pg_run **out);
  * statistics are retrievable with pg_collect_site_stats. */
 int pg_check_banks(const pg_ir *k, const pg_space *sp, pg_run **out);
 
+/* Property mode: check k
+ * against a post-condition given as an IR kernel `post` that computes the expected
+ * outputs from the same inputs (the assertion's quantified equalities become its
+ * loops; subjects/post_*.pgk).  For launch i, k runs with sp->launch_src[i] and post
+ * as one block of one thread whose scalars are the first m (m = post's scalar
+ * count) of (gdim.x, gdim.y, bdim.x, bdim.y, launch_src[i].scalar[0..]).  Then the
+ * comparative assertion of pg_check_equiv (every out/inout array, matched by name)
+ * plus sp->checks on both kernels.  sp->launch_tgt must be NULL (PG_E_ARG); m larger
+ * than the available values is PG_E_ARG. */
+int pg_check_property(const pg_ir *k, const pg_ir *post, const pg_space *sp, pg_run **out);
+
 /* Synchronise the run's stream, copy up to `cap` records (canonical key
  * order) into buf, report how many exist in *n_written (may exceed cap), and
  * fill *sum (may be NULL) from d_first_key / d_counts as they are now. */

@@ -71,7 +71,7 @@ class PgError(RuntimeError):
 
 
 _lib = None
-EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_collect_cex",
+EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
            "pg_collect_site_stats", "pg_collect_dataflow", "pg_ir_info", "pg_ir_source", "pg_ir_compile", "pg_run_timing",
            "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
 
@@ -90,6 +90,7 @@ def lib():
     L.pg_check_equiv.argtypes = [vp, vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_check_races.argtypes = [vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_check_banks.argtypes = [vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
+    L.pg_check_property.argtypes = [vp, vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_collect_cex.argtypes = [vp, ctypes.POINTER(PgCex), ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t),
                                  ctypes.POINTER(PgSummary)]
     L.pg_collect_site_stats.argtypes = [vp, ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32]
@@ -106,7 +107,7 @@ def lib():
     L.pg_version.restype = ctypes.c_char_p
     L.pg_ir_free.argtypes = [vp]
     L.pg_run_free.argtypes = [vp]
-    for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_collect_cex",
+    for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
               "pg_collect_site_stats", "pg_collect_dataflow", "pg_ir_info", "pg_ir_source", "pg_ir_compile",
               "pg_run_timing"):
         getattr(L, f).restype = ctypes.c_int
@@ -282,7 +283,14 @@ def pg_check_banks(k: Ir, space: Space) -> Run:
     return _run(lib().pg_check_banks, [k], space)
 
 
-check_equiv, check_races, check_banks = pg_check_equiv, pg_check_races, pg_check_banks
+def pg_check_property(k: Ir, post: Ir, space: Space) -> Run:
+    """k against the post-condition kernel `post` (one thread per launch; see pgvc.h)."""
+    if space.launch_tgt is not None:
+        raise ValueError("property mode derives the post-condition launches; launch_tgt must be None")
+    return _run(lib().pg_check_property, [k, post], space)
+
+
+check_equiv, check_races, check_banks, check_property = pg_check_equiv, pg_check_races, pg_check_banks, pg_check_property
 
 
 def version() -> str:

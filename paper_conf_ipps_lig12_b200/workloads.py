@@ -205,3 +205,18 @@ def c5_matmul(n_seeds: int = 10000, sizes=(32, 64, 128, 256, 512, 1024), K: int 
     ls = [Launch((N // tile, N // tile, 1), (tile, tile, 1), (K, N, N)) for N in sizes]
     return Workload("C5:matmul", "matmul_naive", tgt, ls, ls, n_seeds=n_seeds,
                     note="naive vs tiled matmul, K = %d" % K)
+
+
+# ---------------------------------------------------------------- property mode (NEXT-1)
+POST = {"reduce": "post_reduce", "scan": "post_scan", "transpose": "post_transpose"}
+
+
+def property_launches(launches: Sequence[Launch], n_post_scalars: int) -> List[Launch]:
+    """The post-condition launches pg_check_property derives (include/pgvc.h): one block of
+    one thread whose scalars are the first m of (gdim.x, gdim.y, bdim.x, bdim.y, scalars)."""
+    out = []
+    for l in launches:
+        v = (l.gdim[0], l.gdim[1], l.bdim[0], l.bdim[1]) + tuple(l.scalars)
+        assert n_post_scalars <= len(v)
+        out.append(Launch((1, 1, 1), (1, 1, 1), tuple(v[:n_post_scalars])))
+    return out

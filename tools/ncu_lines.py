@@ -1,13 +1,24 @@
 """Per-source-line totals (instructions executed, stall samples) of one kernel launch in an
 ncu report captured with --import-source on (uses the correlated cuda,sass source page).
-usage: python tools/ncu_lines.py REPORT [launch_index] [top_n]"""
+usage: python tools/ncu_lines.py REPORT [launch_index] [top_n] [source_dir]
+source_dir: where the NVRTC sources were dumped (PGVC_DUMP_SRC) to print the line text."""
+import os
 import csv
 import io
 import subprocess
 import sys
 
 
-def main(rep, idx=0, top=40):
+def main(rep, idx=0, top=40, srcdir=None):
+    texts = {}
+
+    def text(f, n, fallback):
+        if srcdir and os.path.exists(os.path.join(srcdir, f)):
+            if f not in texts:
+                texts[f] = open(os.path.join(srcdir, f)).read().split("\n")
+            if 0 < n <= len(texts[f]):
+                return texts[f][n - 1].strip()[:90]
+        return fallback
     out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass",
                           "--launch-skip", str(idx), "--launch-count", "1"], capture_output=True, text=True).stdout
     agg, cur, path, hdr = {}, None, "", None
@@ -24,7 +35,7 @@ def main(rep, idx=0, top=40):
             continue
         if not r[0]:      # SASS rows: the source-line row above carries their totals
             continue
-        cur = (path, int(r[0]), r[1].strip()[:90])
+        cur = (path, int(r[0]), text(path, int(r[0]), r[1].strip()[:90]))
         num = lambda x: int(x) if x and x != "-" else 0
         ie, smp = num(r[7]), num(r[4])
         a = agg.setdefault(cur, [0, 0])
@@ -38,4 +49,5 @@ def main(rep, idx=0, top=40):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 0, int(sys.argv[3]) if len(sys.argv) > 3 else 40)
+    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 0, int(sys.argv[3]) if len(sys.argv) > 3 else 40,
+         sys.argv[4] if len(sys.argv) > 4 else None)
