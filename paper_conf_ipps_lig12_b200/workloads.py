@@ -220,3 +220,14 @@ def property_launches(launches: Sequence[Launch], n_post_scalars: int) -> List[L
         assert n_post_scalars <= len(v)
         out.append(Launch((1, 1, 1), (1, 1, 1), tuple(v[:n_post_scalars])))
     return out
+
+
+# ---------------------------------------------------------------- configuration bugs (NEXT-3)
+def scalar_prod_launch(vectorN: int, elementN: int, accn: int, bdim: int) -> Launch:
+    """scalarProd with one vector per block (gdim.x = vectorN), ACCN partial sums."""
+    return Launch((vectorN, 1, 1), (bdim, 1, 1), (vectorN, elementN, accn))
+
+
+def accn_sweep(max_accn: int = 16, bdims=(1, 4, 8), vectorN: int = 2, elementN: int = 40) -> List[Launch]:
+    """ACCN = 1..max_accn in order (the witness order), for each block size."""
+    return [scalar_prod_launch(vectorN, elementN, a, b) for a in range(1, max_accn + 1) for b in bdims]

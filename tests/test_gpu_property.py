@@ -8,7 +8,7 @@ from test_gpu_parity import assert_same
 
 pytestmark = pytest.mark.gpu
 
-POST_SCALARS = {"post_reduce": 5, "post_scan": 5, "post_transpose": 6}
+POST_SCALARS = {"post_reduce": 5, "post_scan": 5, "post_transpose": 6, "post_scalar_prod": 6}
 
 
 @pytest.fixture(scope="module")
