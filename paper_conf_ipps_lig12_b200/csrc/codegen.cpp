@@ -12,6 +12,8 @@
 //     warp-level bank / coalescing intrinsics see the whole warp.
 // Loads are predicated (short-circuit && || ?: keep their guards, X2/X21).
 #include <cstdio>
+#include <map>
+#include <set>
 #include <sstream>
 
 #include "front.hpp"
@@ -90,6 +92,91 @@ struct Gen {
         }
     }
 
+    // ---------------------------------------------------------------- round-segment analysis
+    // Barriers are block-uniform (X18), so in one round every thread of a block runs code
+    // entered from the same barrier.  For each program point: the set of barriers (nullptr =
+    // kernel entry) from which it is reachable without crossing another barrier.  A load of
+    // an array needs reader stamps only if some store to that array shares a barrier with
+    // it: otherwise no write of the array can fall in the load's round (no RW race, X4).
+    using SegSet = std::set<const Stmt*>;
+    std::map<const Node*, SegSet> seg_ld_;
+    std::vector<SegSet> seg_st_;
+    bool seg_changed_ = false;
+    static bool merge_into(SegSet& dst, const SegSet& src) {
+        size_t n = dst.size();
+        dst.insert(src.begin(), src.end());
+        return dst.size() != n;
+    }
+    void seg_expr(const Node* n, const SegSet& st) {
+        if (!n) return;
+        for (const Node* k : n->kids) seg_expr(k, st);
+        if (n->kind == NK::Elem) seg_changed_ |= merge_into(seg_ld_[n], st);
+    }
+    void seg_stmt(const Stmt* s, SegSet& st) {
+        if (!s) return;
+        switch (s->kind) {
+        case SK::Seq:
+            for (const Stmt* c : s->seq) seg_stmt(c, st);
+            break;
+        case SK::Assign: seg_expr(s->value, st); break;
+        case SK::Store:
+            for (const Node* i : s->index) seg_expr(i, st);
+            seg_expr(s->value, st);
+            seg_changed_ |= merge_into(seg_st_[(size_t)s->arr], st);
+            break;
+        case SK::PrivDecl:
+            for (const Node* i : s->index) seg_expr(i, st);
+            seg_expr(s->value, st);
+            break;
+        case SK::Sync: st = SegSet{s}; break;
+        case SK::If: {
+            seg_expr(s->cond, st);
+            SegSet a = st, b = st;
+            seg_stmt(s->body, a);
+            seg_stmt(s->other, b);
+            st = a;
+            merge_into(st, b);
+            break;
+        }
+        case SK::Loop: {
+            // conservative: the head sees its entry and every state inside the loop (covers
+            // back edges, continue and break); iterate to a fixed point
+            seg_stmt(s->init, st);
+            SegSet head = st;
+            for (;;) {
+                SegSet in = head, all = head;
+                seg_expr(s->cond, in);
+                seg_stmt(s->body, in);
+                merge_into(all, in);
+                seg_stmt(s->step, in);
+                merge_into(all, in);
+                if (!merge_into(head, all)) break;
+            }
+            seg_expr(s->cond, head);
+            st = head;
+            break;
+        }
+        default: break;
+        }
+    }
+    void seg_run() {
+        seg_st_.assign(K.arrays.size(), SegSet());
+        do {
+            seg_changed_ = false;
+            SegSet st{nullptr};
+            seg_stmt(K.body, st);
+        } while (seg_changed_);
+    }
+    // reader stamps for this load site
+    bool stamps_needed(const Node* n) const {
+        if (!reader_tracked(n->ref)) return false;
+        auto it = seg_ld_.find(n);
+        if (it == seg_ld_.end()) return true;
+        for (const Stmt* b : it->second)
+            if (seg_st_[(size_t)n->ref].count(b)) return true;
+        return false;
+    }
+
     Gen(const Kernel& k, const CodegenOptions& o) : K(k), O(o) {
         mask = o.bits >= 32 ? 0xFFFFFFFFu : ((1u << o.bits) - 1u);
     }
@@ -123,6 +210,7 @@ struct Gen {
         for (size_t k = 1; k < iv.size(); k++) {
             std::string dim;
             if (a.space == PRIVATE) dim = hex(a.dims[k]->lit);
+            else if (a.space == SHARED) dim = "PG_SH(" + std::to_string(arr) + ", d" + std::to_string(k) + ")";
             else dim = "pg_sL.arr[" + std::to_string(arr) + "].d" + std::to_string(k);
             line(f + " = " + f + " * " + dim + " + " + iv[k] + ";");
         }
@@ -147,11 +235,11 @@ struct Gen {
             std::string r = tmp();
             std::string A = std::to_string(n->ref), S = std::to_string(n->site) + "u";
             if (a.space == SHARED) {
-                line("u32 " + r + " = pg_ld_sh<" + A + ", " + (reader_tracked(n->ref) ? "true" : "false") + ", " +
+                line("u32 " + r + " = pg_ld_sh<" + A + ", " + (stamps_needed(n) ? "true" : "false") + ", " +
                      (log_[(size_t)n->ref] ? "true" : "false") + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
             } else if (a.space == GLOBAL) {
                 if (a.written)
-                    line("u32 " + r + " = pg_ld_gt<" + A + ", " + (reader_tracked(n->ref) ? "true" : "false") + ", " +
+                    line("u32 " + r + " = pg_ld_gt<" + A + ", " + (stamps_needed(n) ? "true" : "false") + ", " +
                          (log_[(size_t)n->ref] ? "true" : "false") + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
                 else
                     line("u32 " + r + " = pg_ld_gi<" + A + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
@@ -410,6 +498,7 @@ struct Gen {
             std::vector<bool> st(K.arrays.size(), false);
             lw_stmt(K.body, st);
         }
+        seg_run();
         stmt(K.body);
         line("t.live = 0u; return PG_END;");
         std::ostringstream o;
