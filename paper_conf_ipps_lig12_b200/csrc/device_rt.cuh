@@ -815,6 +815,8 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     __shared__ u64 s_part[32];   // per-warp instance counts
     __syncthreads();
     const bool grid_1d = pg_sL.gdim[1] == 1u && pg_sL.gdim[2] == 1u;
+    const bool grid_pow2 = !(pg_sL.gdim[0] & (pg_sL.gdim[0] - 1u)) && !(pg_sL.gdim[1] & (pg_sL.gdim[1] - 1u));
+    const u32 gsh0 = __ffs(pg_sL.gdim[0]) - 1, gsh1 = __ffs(pg_sL.gdim[1]) - 1;
     u64 inst = 0;  // instances of this group (accumulated by its lane tl0 == 0)
     const u32 nsteps = (pg_sW.blk1 - pg_sW.blk0 + GB - 1) / GB;
     for (u32 st = 0; st < nsteps; st++) {
@@ -830,6 +832,10 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             if (grid_1d) {
                 t.bid[0] = blk;
                 t.bid[1] = t.bid[2] = 0u;
+            } else if (grid_pow2) {   // (power-of-two grid dims: shifts instead of divisions)
+                t.bid[0] = blk & (pg_sL.gdim[0] - 1u);
+                t.bid[1] = (blk >> gsh0) & (pg_sL.gdim[1] - 1u);
+                t.bid[2] = blk >> (gsh0 + gsh1);
             } else {
                 t.bid[0] = blk % pg_sL.gdim[0];
                 t.bid[1] = (blk / pg_sL.gdim[0]) % pg_sL.gdim[1];
@@ -891,8 +897,9 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             __syncwarp();
             if (inst_ok && tl0 == 0u) s_grounds[g] = 0u;
             __syncwarp();
-        } else {
-            if (inst_ok && alive_rounds) atomicMax(&s_grounds[g], alive_rounds);
+        } else {   // a warp lies in one group: warp max, then one shared atomic per warp
+            const u32 wm = __reduce_max_sync(PG_FULL, inst_ok ? alive_rounds : 0u);
+            if (lane == 0u && inst_ok && wm) atomicMax(&s_grounds[g], wm);
             __syncthreads();
             grounds = inst_ok ? s_grounds[g] : 0u;
             __syncthreads();

@@ -44,7 +44,8 @@ def main(rep, idx=0, top=40, srcdir=None):
     ti = sum(a[0] for a in agg.values()) or 1
     ts = sum(a[1] for a in agg.values()) or 1
     print("instructions %d, samples %d" % (ti, ts))
-    for k, a in sorted(agg.items(), key=lambda kv: -kv[1][0])[:top]:
+    key = 1 if os.environ.get("SORT_SAMPLES") else 0
+    for k, a in sorted(agg.items(), key=lambda kv: -kv[1][key])[:top]:
         print("%6.2f%% ins %6.2f%% smp  %s:%d  %s" % (100 * a[0] / ti, 100 * a[1] / ts, k[0], k[1], k[2]))
 
 

@@ -5,12 +5,13 @@
 #   3. one `--set full` capture of the top evaluation-kernel launch (source-level, -lineinfo)
 set -u
 OUT=${1:-gpurun_out/prof}
+WL=${2:-c2}
 mkdir -p "$OUT/src"
 ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start off --csv \
-    --log-file "$OUT/launches.csv" python bench.py --profile > "$OUT/launches.log" 2>&1
+    --log-file "$OUT/launches.csv" python bench.py --profile --workload "$WL" > "$OUT/launches.log" 2>&1
 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__warps_active.avg.pct_of_peak_sustained_active,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active \
     --clock-control none --profile-from-start off -k regex:pgk_eval --csv \
-    --log-file "$OUT/k2_metrics.csv" python bench.py --profile > "$OUT/k2_metrics.log" 2>&1
+    --log-file "$OUT/k2_metrics.csv" python bench.py --profile --workload "$WL" > "$OUT/k2_metrics.log" 2>&1
 # the longest evaluation-kernel launch of the metrics pass (same filter => same launch index)
 SKIP=${K2_SKIP:-$(python - "$OUT/k2_metrics.csv" <<'PY'
 import csv, sys
@@ -28,5 +29,5 @@ PY
 )}
 echo "k2 top launch index: $SKIP"
 PGVC_DUMP_SRC="$PWD/$OUT/src" ncu --set full --clock-control none --import-source on --profile-from-start off \
-    -k regex:pgk_eval -s "$SKIP" -c 1 -o "$OUT/k2_top" python bench.py --profile > "$OUT/k2_top.log" 2>&1
+    -k regex:pgk_eval -s "$SKIP" -c 1 -o "$OUT/k2_top" python bench.py --profile --workload "$WL" > "$OUT/k2_top.log" 2>&1
 echo done
