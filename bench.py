@@ -129,14 +129,15 @@ def measured_peaks():
         return {}
 
 
-def ncu_traffic():
-    """Per-launch DRAM bytes of the evaluation kernel from the committed ncu capture (or None)."""
-    p = os.path.join(ROOT, "profiles", "r1", "k2_traffic.json")
+def ncu_profile():
+    """The committed ncu summary of the evaluation kernel for this workload ({} if none):
+    profiles/r1/k2_traffic.json for C2, profiles/r1/<workload>/k2_traffic.json otherwise."""
+    p = os.path.join(ROOT, "profiles", "r1", *(() if WL == "c2" else (WL,)), "k2_traffic.json")
     try:
         with open(p) as f:
-            return json.load(f).get("bytes_per_launch")
+            return json.load(f)
     except (OSError, ValueError):
-        return None
+        return {}
 
 
 # ---------------------------------------------------------------- CPU oracle (reference arm / cpu_baseline)
@@ -358,7 +359,9 @@ def main():
                    "parallelism": "dp%d over seeds" % world},
         "roofline": {"bound": "alu", "achieved": achieved_ops / 1e12 if achieved_ops else None,
                      "peak": alu_peak / 1e12, "unit": "Tops/s (int32, algorithmic IR ops)",
-                     "frac": (achieved_ops / alu_peak) if achieved_ops else None, "traffic": ncu_traffic(),
+                     "frac": (achieved_ops / alu_peak) if achieved_ops else None,
+                     "traffic": ncu_profile().get("bytes_per_launch"),
+                     "ncu_issue_active_pct": ncu_profile().get("issue_active_pct_time_weighted"),
                      "kernel": "pgk_eval (K2)", "ops_per_instance": OPS_PER_INSTANCE,
                      "k2_ms_per_step": eval_ms / args.steps,
                      "peak_source": "148 SM x 64 int32 lanes/clk x sm_max_mhz (DESIGN.md §6)"},

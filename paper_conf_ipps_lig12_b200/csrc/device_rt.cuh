@@ -796,7 +796,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     for (u32 v = 0; v < PG_VMAX; v++) {
         if (v >= V) break;
         PgT& t = T[v];
-        t.tlin = tl0 + v * 1024u;
+        t.tlin = tl0 + v * (32u * PG_WPG);   // virtual thread v: lanes of the v-th slice of the block
         const u32 ok = inst_ok && t.tlin < T_;
         t.ekey = ok ? ekey : 63u;
         t.lane = lane;

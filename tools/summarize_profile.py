@@ -23,9 +23,10 @@ def num(x):
     return float(x.replace(",", ""))
 
 
-def main(src, dst):
+def main(src, dst, workload="c2"):
     os.makedirs(dst, exist_ok=True)
-    lines = ["# ncu summary (one bench step of the headline workload, C2)", ""]
+    lines = ["# ncu summary: one bench step of workload %s (`tools/profile_round.sh OUT %s`)" % (workload, workload), "",
+             "ncu times are cold-cache and serialised (compare shares, not absolute times).", ""]
     L = rows(os.path.join(src, "launches.csv"))
     agg = collections.defaultdict(lambda: [0, 0.0])
     for d in L:
@@ -72,6 +73,14 @@ def main(src, dst):
             "Grid Size", "Dynamic Shared"))]
         lines += ["## Top evaluation-kernel launch (`--set full`)", "", "```"] + keep + ["```", ""]
         shutil.copy(rep, os.path.join(dst, "k2_top.ncu-rep"))
+        # where the top launch's instructions and stall samples go, per source line
+        here = os.path.dirname(os.path.abspath(__file__))
+        for title, env in (("instructions executed", {}), ("stall samples", {"SORT_SAMPLES": "1"})):
+            out = subprocess.run([sys.executable, os.path.join(here, "ncu_lines.py"), os.path.abspath(rep), "0", "15",
+                                  os.path.abspath(os.path.join(src, "src"))], capture_output=True, text=True,
+                                 cwd="/", env=dict(os.environ, **env)).stdout
+            lines += ["### Top source lines by %s" % title, "", "```"] + \
+                [l[:150] for l in out.splitlines()] + ["```", ""]
     shutil.copy(os.path.join(src, "launches.csv"), os.path.join(dst, "launches.csv"))
     shutil.copy(os.path.join(src, "k2_metrics.csv"), os.path.join(dst, "k2_metrics.csv"))
     open(os.path.join(dst, "SUMMARY.md"), "w").write("\n".join(lines) + "\n")
@@ -79,4 +88,4 @@ def main(src, dst):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2])
+    main(sys.argv[1], sys.argv[2], sys.argv[3] if len(sys.argv) > 3 else "c2")
