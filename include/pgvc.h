@@ -137,9 +137,10 @@ int pg_check_banks(const pg_ir *k, const pg_space *sp, pg_run **out);
  * than the available values is PG_E_ARG. */
 int pg_check_property(const pg_ir *k, const pg_ir *post, const pg_space *sp, pg_run **out);
 
-/* Synchronise the run's stream, copy up to `cap` records (canonical key
- * order) into buf, report how many exist in *n_written (may exceed cap), and
- * fill *sum (may be NULL) from d_first_key / d_counts as they are now. */
+/* Synchronise the run's stream, copy the first min(*n_written, cap, max_cex)
+ * records (canonical key order; the run keeps at most pg_space.max_cex, 0 =
+ * 2^20) into buf, report how many exist in *n_written (may exceed both caps),
+ * and fill *sum (may be NULL) from d_first_key / d_counts as they are now. */
 int pg_collect_cex(pg_run *r, pg_cex *buf, size_t cap, size_t *n_written, pg_summary *sum);
 
 /* Per-site bank/coalescing statistics of a run: uint64

@@ -226,7 +226,7 @@ class Run:
         buf = np.empty(max(1, cap), dtype=REC_DTYPE)
         _ck(lib().pg_collect_cex(self._h, buf.ctypes.data_as(ctypes.POINTER(PgCex)), cap, ctypes.byref(n),
                                  ctypes.byref(summ)))
-        arr = buf[:min(n.value, cap)]
+        arr = buf[:min(n.value, cap, self.space.max_cex or (1 << 20))]   # the run keeps max_cex
         recs = arr.tolist() if tuples else arr
         s = {"instances": summ.instances, "n_fail": summ.n_fail, "n_records": summ.n_records,
              "first_key": summ.first_key, "first_launch": summ.first_launch,
