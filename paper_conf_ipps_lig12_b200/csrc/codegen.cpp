@@ -45,6 +45,7 @@ struct Gen {
     std::vector<std::string> preds;  // thread-dependent predicate variables, innermost last
     std::vector<Loop> loops;
     std::vector<bool> log_;          // per array: a load may follow the thread's own store in one round
+    bool inline_ = false;            // emitting `run` (rounds inline) rather than the re-entrant `seg`
 
     // ---------------------------------------------------------------- own-write analysis
     // Conservative flow walk: which arrays may have been stored by this thread since
@@ -365,13 +366,17 @@ struct Gen {
             return;
         case SK::Sync: {
             int k = ++nsync;
+            if (inline_) {   // end this round in place; stop when every thread has exited
+                line("if (!pg_round_end<PgK, false>(C, t, c, ar)) return;");
+                return;
+            }
             line("return " + std::to_string(k) + "u;");
             body << "R" << k << ":;\n";
             return;
         }
         case SK::Return:
             if (uniform_ctx()) {
-                line("t.live = 0u; return PG_END;");
+                line(inline_ ? "t.live = 0u; goto PG_DONE;" : "t.live = 0u; return PG_END;");
             } else {
                 line("{");
                 line("const u32 _k = " + eff() + ";");
@@ -451,7 +456,8 @@ struct Gen {
         if (s->step) stmt(s->step);
         loops.pop_back();
         line("pg_tick(C, t, c, t.live);");
-        line("if (++C.ufuel > C.fuel) { t.live = 0u; return PG_END; }");
+        line(inline_ ? "if (++C.ufuel > C.fuel) { t.live = 0u; goto PG_DONE; }"
+                     : "if (++C.ufuel > C.fuel) { t.live = 0u; return PG_END; }");
         line("goto L" + std::to_string(head) + ";");
         body << "L" << L.exit_label << ":;\n";
     }
@@ -499,8 +505,27 @@ struct Gen {
             lw_stmt(K.body, st);
         }
         seg_run();
-        stmt(K.body);
-        line("t.live = 0u; return PG_END;");
+        // the body twice: `seg` (re-entrant at every barrier; virtual-thread variants) and
+        // `run` (a whole block, rounds ended in place)
+        auto emit = [&](bool inl) {
+            ntmp = nlabel = nsync = 0;
+            body.str("");
+            preds.clear();
+            loops.clear();
+            inline_ = inl;
+            stmt(K.body);
+            if (inl) {
+                line("t.live = 0u;");
+                body << "PG_DONE:;\n";
+                line("pg_round_end<PgK, true>(C, t, c, ar);");
+            } else {
+                line("t.live = 0u; return PG_END;");
+            }
+            return body.str();
+        };
+        const std::string seg_body = emit(false);
+        const int seg_nsync = nsync;
+        const std::string run_body = emit(true);
         std::ostringstream o;
         o << "#define PG_BITS " << O.bits << "\n";
         o << "#define PG_RACECHK " << ((O.checks & 2) ? 1 : 0) << "\n";
@@ -550,9 +575,12 @@ struct Gen {
         o << "      default: break;\n    }\n  }\n";
         o << "  static __device__ __forceinline__ u32 seg(Frame& F, PgC& C, PgT& t, PgCold& c, u64* ss, u32 resume) {\n";
         o << "    switch (resume) {\n      case 0u: goto R0;\n";
-        for (int k = 1; k <= nsync; k++) o << "      case " << k << "u: goto R" << k << ";\n";
+        for (int k = 1; k <= seg_nsync; k++) o << "      case " << k << "u: goto R" << k << ";\n";
         o << "      default: return PG_END;\n    }\n";
-        o << "R0:;\n" << body.str();
+        o << "R0:;\n" << seg_body;
+        o << "  }\n";
+        o << "  static __device__ __forceinline__ void run(Frame& F, PgC& C, PgT& t, PgCold& c, u64* ss, u32& ar) {\n";
+        o << run_body;
         o << "  }\n};\n\n";
         o << "#ifndef PG_CTA_MAX\n#define PG_CTA_MAX 1024\n#define PG_MIN_BLOCKS 1\n#endif\n";
         o << "extern \"C\" __global__ void __launch_bounds__(PG_CTA_MAX, PG_MIN_BLOCKS) pgk_eval(const PgParams P) "

@@ -574,6 +574,28 @@ __device__ __forceinline__ void pg_check_all(const PgC& C, const PgT& t, PgCold&
     for (u32 i = 1; i < t.nlog; i++) K::check_one(C, t, c, c.lcell[i], c.lval[i], c.lsite[i]);
 }
 
+// End of a round when the rounds of a block run inline (K::run, one emulated thread
+// per lane): barrier, claims, barrier, checks, then the early-exit vote.  Unless LAST,
+// begin the next round and return whether any thread of the CTA is still live.
+template <class K, bool LAST>
+__device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& alive_rounds) {
+    const bool warp_blocks = PG_T <= 32u;
+    if (warp_blocks) __syncwarp(); else __syncthreads();
+    pg_claim_all<K>(C, t, c);
+    if (warp_blocks) __syncwarp(); else __syncthreads();
+    pg_check_all<K>(C, t, c);
+    C.round++;
+    if (LAST) return false;
+    const int more = warp_blocks ? __any_sync(PG_FULL, t.live) : __syncthreads_or((int)t.live);
+    if (!more) return false;
+    C.step++;
+    C.ufuel = 0;
+    t.nlog = 0;
+    t.fuel = 0;
+    alive_rounds += t.live;
+    return true;
+}
+
 // ------------------------------------------------------------------ records (H8)
 // Each thread keeps its minimum event per kind.  At the end of the CTA: (1) the
 // lanes of a warp that belong to the same instance merge (lexicographic min by
@@ -849,6 +871,17 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         if (pg_sL.off_step0 != ~0ull && inst_ok && tl0 == 0u && blk_ok) T[0].arena[pg_sL.off_step0 + blk] = C.step0;
 #endif
         C.round = 0;
+#if PG_VMAX == 1
+        {   // rounds inline: K::run ends each round at its barrier (pg_round_end)
+            PgT& t = T[0];
+            C.step++;
+            C.ufuel = 0;
+            t.nlog = 0;
+            t.fuel = 0;
+            alive_rounds = t.live;
+            K::run(F[0], C, t, Cd[0], sstats, alive_rounds);
+        }
+#else
         u32 resume = 0;
         for (;;) {
             C.step++;
@@ -883,6 +916,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             if (r == PG_END || !more) break;
             resume = r;
         }
+#endif
         // rounds of this group's block = max over its threads of the rounds they entered alive
         u32 grounds;
         if (warp_blocks && (T_ & (T_ - 1u)) == 0u) {
