@@ -84,6 +84,10 @@ def lib():
             _lib.or_dataflow.argtypes = [ctypes.c_char_p, ctypes.POINTER(OrLaunch), ctypes.c_uint64,
                                          ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32), ctypes.c_uint64,
                                          ctypes.POINTER(ctypes.c_uint64)]
+            _lib.or_lockstep.restype = ctypes.c_int
+            _lib.or_lockstep.argtypes = [ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(OrSpace), ctypes.c_uint32,
+                                         ctypes.POINTER(ctypes.c_uint32), ctypes.c_uint64,
+                                         ctypes.POINTER(ctypes.c_uint64)]
             _lib.or_last_error.restype = ctypes.c_char_p
             _lib.or_sm64.restype = ctypes.c_uint64
             _lib.or_sm64.argtypes = [ctypes.c_uint64]
@@ -180,6 +184,33 @@ def exec_kernel(text: str, launch, seed: int, *, input_mode=0, input_range=0, bi
         a_fin.append(af[off:off + n].copy())
         off += n
     return a_init, a_fin, list(counts)
+
+
+LOCK_FIELDS = ("launch", "seed_idx", "block", "round", "array", "addr", "val_src", "val_tgt", "written_src",
+               "written_tgt")
+
+
+def lockstep(src: str, tgt: str, launch_src, launch_tgt=None, *, lock_rounds=32, n_seeds=1, seed_base=0,
+             input_mode=0, input_range=0, bits=32, cap=1 << 16):
+    """Lock-step comparison of a pair (X25): per instance, the first (block, round,
+    array, addr) at which the kernels' shared contents differ; rows of LOCK_FIELDS."""
+    L = lib()
+    ls = _launch_array(launch_src)
+    lt = _launch_array(launch_tgt) if launch_tgt is not None else None
+    sp = OrSpace()
+    sp.launch_src = ctypes.cast(ls, ctypes.POINTER(OrLaunch))
+    sp.launch_tgt = ctypes.cast(lt, ctypes.POINTER(OrLaunch)) if lt is not None else None
+    sp.n_launch = len(launch_src)
+    sp.seed_base, sp.n_seeds, sp.rank, sp.world = seed_base, n_seeds, 0, 1
+    sp.input_mode, sp.input_range, sp.bits = input_mode, input_range, bits
+    sp.checks, sp.wmax, sp.mode = EQUIV | RACE | OOB, 32, MODE_EQUIV
+    rows = (ctypes.c_uint32 * (cap * 10))()
+    n = ctypes.c_uint64(0)
+    rc = L.or_lockstep(src.encode(), tgt.encode(), ctypes.byref(sp), lock_rounds, rows, cap, ctypes.byref(n))
+    if rc != 0:
+        raise OracleError(rc, L.or_last_error().decode())
+    a = np.ctypeslib.as_array(rows)[: min(n.value, cap) * 10].reshape(-1, 10)
+    return [tuple(int(x) for x in r) for r in a]
 
 
 DF_FIELDS = ("block", "round", "gtid", "site", "array", "addr", "src_kind", "w_block", "w_round", "w_gtid")

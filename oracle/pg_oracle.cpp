@@ -1009,6 +1009,7 @@ struct Config {
     uint64_t fuel = 1u << 20;
     bool vcliteral = false;
     bool dataflow = false;
+    uint32_t lock_rounds = 0;   /* lock-step comparison: snapshot rounds < lock_rounds (0: off) */
 };
 
 struct DFRow {   /* data-flow relation row (H5): who supplied the value of a read */
@@ -1111,6 +1112,17 @@ static uint32_t eval_uniform(const Kernel& K, const Expr* e, const Launch& L) {
     return ev(e);
 }
 
+/* Lock-step comparison (X25): the contents of
+ * one shared array of one block after one round, as (written << 32) | value. */
+struct Snap {
+    uint32_t block, round;
+    std::string name;
+    std::vector<uint64_t> cells;
+};
+struct DivRow {   /* first divergence of an instance: block, round, array, addr, values, written flags */
+    uint32_t launch, seed_idx, block, round, array, addr, val_s, val_t, wr_s, wr_t;
+};
+
 struct Results {
     /* slots[(launch, seed_j, kernel)][kind] */
     std::map<std::tuple<uint32_t, uint32_t, uint32_t>, SlotSet> slots;
@@ -1118,6 +1130,8 @@ struct Results {
     std::vector<uint64_t> site_stats;   /* [n_launch][2][max_sites][8] */
     uint32_t max_sites = 0;
     std::vector<DFRow> df;
+    std::vector<Snap> snaps[2];      /* per kernel, this instance */
+    std::vector<DivRow> div;
 };
 
 /* Executes one kernel for one (launch, seed); returns final global memory. */
@@ -1581,6 +1595,18 @@ struct Exec {
                 }
                 commit_round();
                 bank_stats();
+                if (cur_round < cfg.lock_rounds) {   /* X25: shared state after this round */
+                    for (size_t a = 0; a < K.arrs.size(); a++) {
+                        const Arr& A = K.arrs[a];
+                        if (A.space != SP_SHARED) continue;
+                        Snap sn;
+                        sn.block = b; sn.round = cur_round; sn.name = A.name;
+                        const size_t li = (size_t)A.local_index;
+                        for (uint32_t i = 0; i < size[a]; i++)
+                            sn.cells.push_back(swritten[li][i] ? ((1ull << 32) | sval[li][i]) : 0ull);
+                        res.snaps[kernel_idx].push_back(std::move(sn));
+                    }
+                }
                 if (cfg.vcliteral) {
                     Hist H; H.block = b; H.round = cur_round;
                     for (uint32_t i = 0; i < T; i++) H.logs.push_back(th[i].wlog);
@@ -1637,6 +1663,34 @@ static void check_launch(const Kernel& K, const Launch& L) {
     if (L.n_scalar != K.scalar_vars.size()) throw Error(E_ARG, "scalar count does not match kernel '" + K.name + "'");
 }
 
+/* X25: the first (block, round, array, addr) - array in the source kernel's shared
+ * declaration order - at which the two kernels' shared contents differ, over the
+ * (block, round, array) snapshots both kernels took with the same array name and size. */
+static void lockstep_compare(const Kernel& ks, uint32_t li, uint32_t sj, Results& res) {
+    std::map<std::tuple<uint32_t, uint32_t, std::string>, const Snap*> tgt;
+    for (const Snap& s : res.snaps[1]) tgt[std::make_tuple(s.block, s.round, s.name)] = &s;
+    std::map<std::string, uint32_t> slot;   /* source shared array name -> record array id */
+    for (const Arr& A : ks.arrs)
+        if (A.space == SP_SHARED) slot[A.name] = 0x100u + (uint32_t)A.local_index;
+    bool found = false;
+    DivRow best{};
+    for (const Snap& s : res.snaps[0]) {
+        auto it = tgt.find(std::make_tuple(s.block, s.round, s.name));
+        if (it == tgt.end() || it->second->cells.size() != s.cells.size()) continue;
+        for (uint32_t i = 0; i < s.cells.size(); i++) {
+            uint64_t a = s.cells[i], b = it->second->cells[i];
+            if (a == b) continue;
+            DivRow r{li, sj, s.block, s.round, slot[s.name], i, (uint32_t)a, (uint32_t)b,
+                     (uint32_t)(a >> 32), (uint32_t)(b >> 32)};
+            auto k = [](const DivRow& x) { return std::make_tuple(x.block, x.round, x.array, x.addr); };
+            if (!found || k(r) < k(best)) best = r;
+            found = true;
+            break;   /* later cells of this snapshot are larger in the order */
+        }
+    }
+    if (found) res.div.push_back(best);
+}
+
 static void run_space(const Kernel* ks, const Kernel* kt, const Space& S, Results& res) {
     KInfo ki[2];
     const Kernel* kk[2] = {ks, kt};
@@ -1665,6 +1719,8 @@ static void run_space(const Kernel* ks, const Kernel* kt, const Space& S, Result
             uint64_t seed = S.seed_base + sj;
             std::vector<std::vector<uint32_t>> fin[2], flast[2], fsize[2];
             std::vector<uint32_t> fsz[2];
+            res.snaps[0].clear();
+            res.snaps[1].clear();
             for (int k = 0; k < nk; k++) {
                 Slot* sl = res.slots[std::make_tuple(li, sj, (uint32_t)k)].s;
                 Exec ex(S.cfg, ki[k], *LL[k], seed, li, sj, (uint32_t)k, sl, res);
@@ -1673,6 +1729,7 @@ static void run_space(const Kernel* ks, const Kernel* kt, const Space& S, Result
                 flast[k] = ex.glast;
                 fsz[k] = ex.size;
             }
+            if (nk == 2 && S.cfg.lock_rounds) lockstep_compare(*ks, li, sj, res);
             if (nk == 2 && (S.cfg.checks & CHK_EQUIV)) {
                 /* comparative assertion o_s = o_t (L441-L444, L652-L657) */
                 Slot* sl = res.slots[std::make_tuple(li, sj, 0u)].s;
@@ -1903,6 +1960,45 @@ int or_dataflow(const char* text, const or_launch* launch, uint64_t seed, uint32
         ex.run();
         *n_rows = res.df.size();
         for (size_t i = 0; i < res.df.size() && i < cap_rows; i++) memcpy(rows + i * 10, &res.df[i], sizeof(DFRow));
+        return 0;
+    } catch (const orc::Error& e) {
+        or_err = e.what();
+        return e.code;
+    } catch (const std::exception& e) {
+        or_err = e.what();
+        return -1;
+    }
+}
+
+/* Lock-step comparison of a pair (X25): for every
+ * instance of the space, the first divergence of the kernels' shared contents after
+ * rounds < lock_rounds, as rows of 10 words [launch, seed_idx, block, round, array,
+ * addr, val_src, val_tgt, written_src, written_tgt] in (launch, seed) order. */
+int or_lockstep(const char* src, const char* tgt, const or_space* sp, uint32_t lock_rounds, uint32_t* rows,
+                uint64_t cap_rows, uint64_t* n_rows) {
+    using namespace orc;
+    try {
+        if (!src || !tgt || !sp || !n_rows) throw Error(E_ARG, "null argument");
+        std::unique_ptr<Kernel> ks = parse_kernel(src), kt = parse_kernel(tgt);
+        Space S;
+        S.launch_src = reinterpret_cast<const Launch*>(sp->launch_src);
+        S.launch_tgt = reinterpret_cast<const Launch*>(sp->launch_tgt);
+        S.n_launch = sp->n_launch;
+        S.seed_base = sp->seed_base;
+        S.n_seeds = sp->n_seeds;
+        S.rank = sp->rank;
+        S.world = sp->world ? sp->world : 1;
+        S.cfg.bits = sp->bits ? sp->bits : 32;
+        S.cfg.input_mode = sp->input_mode;
+        S.cfg.input_range = sp->input_range;
+        S.cfg.checks = sp->checks;
+        S.cfg.wmax = sp->wmax ? sp->wmax : 32;
+        S.cfg.lock_rounds = lock_rounds;
+        S.mode = sp->mode;
+        Results res;
+        run_space(ks.get(), kt.get(), S, res);
+        *n_rows = res.div.size();
+        for (size_t i = 0; i < res.div.size() && i < cap_rows; i++) memcpy(rows + i * 10, &res.div[i], sizeof(DivRow));
         return 0;
     } catch (const orc::Error& e) {
         or_err = e.what();
