@@ -49,7 +49,9 @@ enum {
 
 enum { PG_IN_RAND32 = 0, PG_IN_BITS01 = 1, PG_IN_RANGE = 2 };                 /* X8 */
 enum { PG_CHK_EQUIV = 1, PG_CHK_RACE = 2, PG_CHK_OOB = 4, PG_CHK_BANK = 8, PG_CHK_COALESCE = 16,
-       PG_CHK_DATAFLOW = 32 /* record the writer of every read (H5); evaluates blocks in bid order */ };
+       PG_CHK_DATAFLOW = 32, /* record the writer of every read (H5); evaluates blocks in bid order */
+       PG_CHK_LOCKSTEP = 64  /* pg_check_equiv: compare the kernels' shared state round by round */ };
+enum { PG_LOCK_ROUNDS = 32 };   /* rounds of every block the lock-step comparison covers */
 enum { PG_BANKS_32 = 0, PG_BANKS_16_HALFWARP = 1 };                             /* X9 */
 enum {                                                                          /* X17 */
     PG_CEX_BARRIER_DIV = 0, PG_CEX_OOB = 1, PG_CEX_RACE_WW = 2, PG_CEX_RACE_RW = 3, PG_CEX_RACE_XB = 4,
@@ -156,6 +158,18 @@ int pg_collect_site_stats(pg_run *r, uint64_t *buf, uint32_t max_sites);
  * w_block, w_round, w_gtid] (0xFFFFFFFF for initial), in no particular order.
  * *n_rows receives the number of reads (rows beyond the capacity are dropped). */
 int pg_collect_dataflow(pg_run *r, uint32_t *rows, size_t cap_rows, size_t *n_rows);
+
+/* Lock-step comparison (X25) of a run checked by
+ * pg_check_equiv with PG_CHK_LOCKSTEP: for the shared arrays both kernels declare
+ * with the same name and size (and launches with the same number of blocks), the
+ * contents after every round < PG_LOCK_ROUNDS of every block are compared.  One row
+ * per instance whose shared states diverge, at the first (block, round, array, addr)
+ * (array in the source kernel's declaration order): 10 x uint32 = [launch, seed_idx,
+ * block, round, array (0x100 + source shared index), addr, val_src, val_tgt,
+ * written_src, written_tgt], in (launch, seed) order; *n_rows = their number.
+ * Blocks of more than 1024 threads are PG_E_LIMIT in this mode; PG_E_STATE if the run
+ * was not checked with PG_CHK_LOCKSTEP. */
+int pg_collect_lockstep(pg_run *r, uint32_t *rows, size_t cap_rows, size_t *n_rows);
 
 /* Introspection of a loaded kernel. */
 int pg_ir_info(const pg_ir *k, uint32_t *n_sites, uint32_t *n_globals, uint32_t *n_scalars);

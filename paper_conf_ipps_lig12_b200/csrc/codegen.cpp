@@ -534,6 +534,7 @@ struct Gen {
         o << "#define PG_COALCHK " << ((O.checks & 16) ? 1 : 0) << "\n";
         o << "#define PG_BANK16 " << (O.bank_model == 1 ? 1 : 0) << "\n";
         o << "#define PG_DATAFLOW " << ((O.checks & 32) ? 1 : 0) << "\n";
+        o << "#define PG_LOCKSTEP " << ((O.checks & 64) ? 1 : 0) << "\n";
         o << "#define PG_WMAX " << O.wmax << "\n";
         o << "#define PG_NSTATS " << std::max<size_t>(1, K.sites.size()) << "\n";
         o << "#ifndef PG_VMAX\n#define PG_VMAX 1\n#endif\n";

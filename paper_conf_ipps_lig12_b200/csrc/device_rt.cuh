@@ -74,6 +74,7 @@ __shared__ PgLaunchK pg_sL;                                 // this CTA's launch
 __shared__ PgWork pg_sW;                                    // this CTA's work item
 
 #define PG_ARR(A) (pg_sL.arr[A])
+#define PG_LOCK_R 32u   // = PG_LOCK_ROUNDS (include/pgvc.h)
 
 // Launch-shape constants.  A variant compiled for one block shape (api.cpp,
 // shape_prelude) defines PG_S_*, and PgSA<A> for the shared-array layout: block
@@ -574,6 +575,26 @@ __device__ __forceinline__ void pg_check_all(const PgC& C, const PgT& t, PgCold&
     for (u32 i = 1; i < t.nlog; i++) K::check_one(C, t, c, c.lcell[i], c.lval[i], c.lsite[i]);
 }
 
+#if PG_LOCKSTEP
+// X25: after the round's commits, every thread of a (real) block copies its share of
+// each matched shared array into the instance's snapshot table.
+__device__ __noinline__ void pg_snapshot(const PgC& C, const PgT& t) {
+    if (t.ekey == 63u || t.blk >= pg_sW.blk1 || C.round >= PG_LOCK_R) return;
+    for (u32 a = 0; a < pg_sL.n_arrays; a++) {
+        const PgArr& R = pg_sL.arr[a];
+        if (R.kind != PGA_SH || R.off_snap == ~0ull) continue;
+        const u32* own = (const u32*)(pg_dsmem + t.sg + R.s_own);
+        const u32* val = (const u32*)(pg_dsmem + t.sg + R.s_val);
+        u32* dst = t.arena + R.off_snap + ((u64)t.blk * PG_LOCK_R + C.round) * R.size * 2u;
+        for (u32 i = t.tlin; i < R.size; i += PG_T) {
+            const u32 w = pg_owner_step(own[i]) >= C.step0;
+            dst[2u * i] = w ? val[i] : 0u;
+            dst[2u * i + 1u] = w;
+        }
+    }
+}
+#endif
+
 // End of a round when the rounds of a block run inline (K::run, one emulated thread
 // per lane): barrier, claims, barrier, checks, then the early-exit vote.  Unless LAST,
 // begin the next round and return whether any thread of the CTA is still live.
@@ -584,6 +605,10 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
     pg_claim_all<K>(C, t, c);
     if (warp_blocks) __syncwarp(); else __syncthreads();
     pg_check_all<K>(C, t, c);
+#if PG_LOCKSTEP
+    if (warp_blocks) __syncwarp(); else __syncthreads();
+    pg_snapshot(C, t);
+#endif
     C.round++;
     if (LAST) return false;
     const int more = warp_blocks ? __any_sync(PG_FULL, t.live) : __syncthreads_or((int)t.live);

@@ -108,6 +108,57 @@ __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ job
     }
 }
 
+// K3b: lock-step comparison (X25).  Per (instance, matched shared array): the smallest
+// (block, round, array, cell) at which both kernels took a snapshot and the (value,
+// written) pairs differ, as key = block << 34 | round << 29 | array << 24 | cell, min-reduced
+// into keys[instance].  Snapshots never taken are all-ones (K1 fill).
+__device__ __forceinline__ u64 pg_lock_key(const PgLock& j, u64 i) {
+    const u64 cell = i % j.size, br = i / j.size;
+    return ((br / j.rounds) << 34) | ((br % j.rounds) << 29) | ((u64)j.arr_slot << 24) | cell;
+}
+__global__ void __launch_bounds__(256) pg_lockstep_cmp(const PgLock* __restrict__ jobs, const u32* arena_s,
+                                                       const u32* arena_t, u64* keys) {
+    const PgLock j = jobs[blockIdx.y];
+    const u64 n = (u64)j.nblocks * j.rounds * j.size;
+    for (u32 inst = blockIdx.x; inst < j.n_inst; inst += gridDim.x) {
+        const uint2* s = (const uint2*)(arena_s + j.src_off + (u64)inst * j.src_stride);
+        const uint2* t = (const uint2*)(arena_t + j.tgt_off + (u64)inst * j.tgt_stride);
+        u64 best = ~0ull;
+        for (u64 i = threadIdx.x; i < n; i += blockDim.x) {   // i order = key order for one array
+            const uint2 a = s[i], b = t[i];
+            if ((a.x & a.y) == PG_NEVER || (b.x & b.y) == PG_NEVER) continue;   // a round one kernel lacks
+            if (a.x != b.x || a.y != b.y) {
+                best = pg_lock_key(j, i);
+                break;
+            }
+        }
+        for (int o = 16; o > 0; o >>= 1) {
+            const u64 x = __shfl_down_sync(0xFFFFFFFFu, best, o);
+            best = x < best ? x : best;
+        }
+        if ((threadIdx.x & 31u) == 0u && best != ~0ull) atomicMin((unsigned long long*)&keys[j.key0 + inst], best);
+    }
+}
+// rows (10 words per instance) for the instances whose minimum lies in this job's array
+__global__ void __launch_bounds__(128) pg_lockstep_fill(const PgLock* __restrict__ jobs, const u32* arena_s,
+                                                        const u32* arena_t, const u64* keys, u32* rows, u32 n_local,
+                                                        u32 rank, u32 world) {
+    const PgLock j = jobs[blockIdx.y];
+    const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
+    if (inst >= j.n_inst) return;
+    const u64 gi = j.key0 + inst, key = keys[gi];
+    if (key == ~0ull || ((key >> 24) & 31u) != j.arr_slot) return;
+    const u64 blk = key >> 34, round = (key >> 29) & 31u, cell = key & 0xFFFFFFu;
+    const u64 i = (blk * j.rounds + round) * j.size + cell;
+    const uint2 a = ((const uint2*)(arena_s + j.src_off + (u64)inst * j.src_stride))[i];
+    const uint2 b = ((const uint2*)(arena_t + j.tgt_off + (u64)inst * j.tgt_stride))[i];
+    u32* r = rows + gi * 10u;
+    r[0] = (u32)(gi / n_local);
+    r[1] = rank + (u32)(gi % n_local) * world;
+    r[2] = (u32)blk; r[3] = (u32)round; r[4] = 0x100u + j.arr_slot; r[5] = (u32)cell;
+    r[6] = a.x; r[7] = b.x; r[8] = a.y; r[9] = b.y;
+}
+
 // K2b': list the sequential-pass items whose seed group has a flagged instance.
 __global__ void __launch_bounds__(256) pg_seq_select(const PgWork* __restrict__ items, u32 n_items,
                                                      const u32* flags, u32* list, u32* count) {
@@ -282,6 +333,18 @@ cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 max_inst, const u32* aren
         pg_compare<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, slots, mm_key);
         dim3 g2((max_inst + 127) / 128, nj);
         pg_compare_fill<<<g2, 128, 0, st>>>(jobs + j0, arena_s, arena_t, input, slots, mm_key);
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t lockstep(const PgLock* jobs, u32 n_jobs, u32 max_inst, const u32* arena_s, const u32* arena_t, u64* keys,
+                     u32* rows, u32 n_local, u32 rank, u32 world, cudaStream_t st) {
+    for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
+        const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
+        dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
+        pg_lockstep_cmp<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, keys);
+        dim3 g2((max_inst + 127) / 128, nj);
+        pg_lockstep_fill<<<g2, 128, 0, st>>>(jobs + j0, arena_s, arena_t, keys, rows, n_local, rank, world);
     }
     return cudaGetLastError();
 }

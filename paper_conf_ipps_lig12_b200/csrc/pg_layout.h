@@ -38,6 +38,8 @@ struct PgArr {
     u64 off_wmax, off_rmin, off_rmax;   // race stamps (~0: absent)
     u64 off_xf, off_xl;                 // first / last accessing block + 1 (~0: absent)
     u64 off_in;     // global arrays the kernel only reads: u32-word offset in the input region
+    u64 off_snap;   // lock-step mode, shared arrays matched in the pair: [block][round < R][cell] x
+                    // (value, written) word pairs in the instance arena (~0: absent)
 };
 
 struct PgLaunchK {
@@ -120,6 +122,15 @@ struct PgXb {
     u64 xf, xl, lw;   // u32-word offsets of instance 0 in the kernel arena
     u64 stride;
     u32 n, n_inst, inst0, pad;
+};
+
+// K3b (pg_lockstep) job: one shared array both kernels of a pair declare (same name
+// and size), snapshotted after rounds < R of every block, for n_inst instances.
+struct PgLock {
+    u64 src_off, tgt_off;        // u32-word offsets of instance 0's snapshots in the two arenas
+    u64 src_stride, tgt_stride;  // arena strides
+    u64 key0;                    // index of instance 0 in the run's per-instance tables
+    u32 n_inst, nblocks, size, rounds, arr_slot, pad;
 };
 
 // K3 (pg_compare) job: one compared global array for n_inst consecutive

@@ -17,7 +17,8 @@ LIB_PATH = os.path.join(_HERE, "libpgvc.so")
 
 PG_OK, PG_E_ARG, PG_E_PARSE, PG_E_TYPE, PG_E_LIMIT, PG_E_CUDA, PG_E_OOM, PG_E_STATE = 0, -1, -2, -3, -4, -5, -6, -7
 IN_RAND32, IN_BITS01, IN_RANGE = 0, 1, 2
-CHK_EQUIV, CHK_RACE, CHK_OOB, CHK_BANK, CHK_COALESCE, CHK_DATAFLOW = 1, 2, 4, 8, 16, 32
+CHK_EQUIV, CHK_RACE, CHK_OOB, CHK_BANK, CHK_COALESCE, CHK_DATAFLOW, CHK_LOCKSTEP = 1, 2, 4, 8, 16, 32, 64
+LOCK_ROUNDS = 32
 BANKS_32, BANKS_16_HALFWARP = 0, 1
 KINDS = ["BARRIER_DIV", "OOB", "RACE_WW", "RACE_RW", "RACE_XB", "MISMATCH", "BANK", "UNCOALESCED", "UNINIT", "LIMIT"]
 N_KINDS = 10
@@ -38,6 +39,8 @@ class PgSpace(ctypes.Structure):
                 ("d_first_key", ctypes.c_void_p), ("d_counts", ctypes.c_void_p)]
 
 
+LOCK_FIELDS = ("launch", "seed_idx", "block", "round", "array", "addr", "val_src", "val_tgt", "written_src",
+               "written_tgt")
 DF_FIELDS = ("launch", "seed_idx", "block", "round", "gtid", "site", "array", "addr", "src", "w_block",
              "w_round", "w_gtid")
 REC_FIELDS = ("key", "count", "kind", "launch", "seed_idx", "kernel", "round", "site", "array", "addr",
@@ -72,8 +75,8 @@ class PgError(RuntimeError):
 
 _lib = None
 EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
-           "pg_collect_site_stats", "pg_collect_dataflow", "pg_ir_info", "pg_ir_source", "pg_ir_compile", "pg_run_timing",
-           "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
+           "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_source",
+           "pg_ir_compile", "pg_run_timing", "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
 
 
 def lib():
@@ -94,6 +97,8 @@ def lib():
     L.pg_collect_cex.argtypes = [vp, ctypes.POINTER(PgCex), ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t),
                                  ctypes.POINTER(PgSummary)]
     L.pg_collect_site_stats.argtypes = [vp, ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32]
+    L.pg_collect_lockstep.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.c_size_t,
+                                      ctypes.POINTER(ctypes.c_size_t)]
     L.pg_collect_dataflow.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.c_size_t,
                                       ctypes.POINTER(ctypes.c_size_t)]
     L.pg_ir_info.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32),
@@ -108,8 +113,8 @@ def lib():
     L.pg_ir_free.argtypes = [vp]
     L.pg_run_free.argtypes = [vp]
     for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
-              "pg_collect_site_stats", "pg_collect_dataflow", "pg_ir_info", "pg_ir_source", "pg_ir_compile",
-              "pg_run_timing"):
+              "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_source",
+              "pg_ir_compile", "pg_run_timing"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -252,6 +257,17 @@ class Run:
                                       ctypes.byref(n)))
         out = out[:min(n.value, 1 << 20)]
         return out[np.lexsort(out.T[::-1])] if len(out) else out
+
+    def lockstep(self):
+        """First shared-state divergence per instance of a PG_CHK_LOCKSTEP equivalence run:
+        list of tuples in LOCK_FIELDS order, (launch, seed) order."""
+        import numpy as np
+        n = ctypes.c_size_t()
+        _ck(lib().pg_collect_lockstep(self._h, None, 0, ctypes.byref(n)))
+        out = np.zeros((max(1, n.value), 10), dtype=np.uint32)
+        _ck(lib().pg_collect_lockstep(self._h, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)), n.value,
+                                      ctypes.byref(n)))
+        return [tuple(int(x) for x in r) for r in out[:n.value]]
 
     def timing(self):
         a, b, n, h = ctypes.c_float(), ctypes.c_float(), ctypes.c_uint32(), ctypes.c_uint64()
