@@ -189,10 +189,14 @@ struct Gen {
     std::string cur() const { return preds.empty() ? std::string("1u") : preds.back(); }
     std::string eff() const { return preds.empty() ? std::string("t.live") : "(" + preds.back() + " & t.live)"; }
 
+    // reader stamps: race checks on, or the optimistic pass (which must detect every race)
     bool reader_tracked(int arr) const {
         const ArrayDecl& a = K.arrays[(size_t)arr];
-        return (O.checks & PG_RACE_BIT) && a.written && a.read && a.space != PRIVATE;
+        return ((O.checks & PG_RACE_BIT) || O.fast) && a.written && a.read && a.space != PRIVATE;
     }
+    // optimistic pass: a store of the array must look for readers of its round
+    std::vector<bool> rda_;
+    std::string rda(int arr) const { return O.fast && rda_[(size_t)arr] ? "true" : "false"; }
     static constexpr uint32_t PG_RACE_BIT = 2;
 
     uint32_t priv_size(const ArrayDecl& a) const {
@@ -340,8 +344,10 @@ struct Gen {
             std::string f = flat_index(&tmpn, s->arr, pe);
             std::string v = ex(s->value, pe);
             std::string A = std::to_string(s->arr), S = std::to_string(s->site) + "u";
-            if (a.space == SHARED) line("pg_st_sh<" + A + ">(C, t, c, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
-            else if (a.space == GLOBAL) line("pg_st_gt<" + A + ">(C, t, c, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
+            if (a.space == SHARED)
+                line("pg_st_sh<" + A + ", " + rda(s->arr) + ">(C, t, c, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
+            else if (a.space == GLOBAL)
+                line("pg_st_gt<" + A + ", " + rda(s->arr) + ">(C, t, c, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
             else
                 line("if (pg_priv_ok(C, t, c, " + pe + ", " + f + ", " + hex(priv_size(a)) + ", " +
                      hex(0x200u + (uint32_t)a.slot) + ", " + S + ", " + v + ", 1u)) F.p" + std::to_string(a.slot) +
@@ -505,6 +511,9 @@ struct Gen {
             lw_stmt(K.body, st);
         }
         seg_run();
+        rda_.assign(K.arrays.size(), false);
+        for (const auto& ld : seg_ld_)
+            if (stamps_needed(ld.first)) rda_[(size_t)ld.first->ref] = true;
         // the body twice: `seg` (re-entrant at every barrier; virtual-thread variants) and
         // `run` (a whole block, rounds ended in place)
         auto emit = [&](bool inl) {
@@ -535,6 +544,7 @@ struct Gen {
         o << "#define PG_BANK16 " << (O.bank_model == 1 ? 1 : 0) << "\n";
         o << "#define PG_DATAFLOW " << ((O.checks & 32) ? 1 : 0) << "\n";
         o << "#define PG_LOCKSTEP " << ((O.checks & 64) ? 1 : 0) << "\n";
+        o << "#define PG_FAST " << (O.fast ? 1 : 0) << "\n";
         o << "#define PG_WMAX " << O.wmax << "\n";
         o << "#define PG_NSTATS " << std::max<size_t>(1, K.sites.size()) << "\n";
         o << "#ifndef PG_VMAX\n#define PG_VMAX 1\n#endif\n";
@@ -564,7 +574,7 @@ struct Gen {
               << ">(C, t, flat); break;\n";
         }
         o << "      default: break;\n    }\n  }\n";
-        o << "  static __device__ __forceinline__ void check_one(const PgC& C, const PgT& t, PgCold& c, u32 cell, "
+        o << "  static __device__ __forceinline__ void check_one(const PgC& C, PgT& t, PgCold& c, u32 cell, "
              "u32 val, u32 site) {\n";
         o << "    const u32 flat = cell & 0xFFFFFFu;\n    switch (cell >> 24) {\n";
         for (size_t a = 0; a < K.arrays.size(); a++) {
@@ -572,6 +582,16 @@ struct Gen {
             if (!A.written || A.space == PRIVATE) continue;
             o << "      case " << a << ": pg_check_" << (A.space == SHARED ? "sh" : "gt") << "<" << a << ", "
               << (reader_tracked((int)a) ? "true" : "false") << ">(C, t, c, flat, val, site); break;\n";
+        }
+        o << "      default: break;\n    }\n  }\n";
+        // optimistic pass: reader check of a logged cell after the round's barrier
+        o << "  static __device__ __forceinline__ void fcheck_one(u32 step, PgT& t, u32 cell) {\n";
+        o << "    const u32 flat = cell & 0xFFFFFFu;\n    switch (cell >> 24) {\n";
+        for (size_t a = 0; a < K.arrays.size(); a++) {
+            const ArrayDecl& A = K.arrays[a];
+            if (!A.written || A.space == PRIVATE || !O.fast || !rda_[a]) continue;
+            o << "      case " << a << ": pg_fcheck_" << (A.space == SHARED ? "sh" : "gt") << "<" << a
+              << ">(step, t, flat); break;\n";
         }
         o << "      default: break;\n    }\n  }\n";
         o << "  static __device__ __forceinline__ u32 seg(Frame& F, PgC& C, PgT& t, PgCold& c, u64* ss, u32 resume) {\n";

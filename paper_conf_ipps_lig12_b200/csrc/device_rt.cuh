@@ -114,6 +114,7 @@ struct PgC {        // CTA-uniform state
     u32 step0;      // step of the first round of the current block
     u32 fuel;
     u32 ufuel;      // uniform-loop iterations this round
+    u32 abort;      // PG_FAST: a race was flagged, the item stops (its instances are re-run exactly)
 };
 
 struct PgT {        // hot per-emulated-thread state (kept in registers)
@@ -123,6 +124,8 @@ struct PgT {        // hot per-emulated-thread state (kept in registers)
     u32 tlin, gtid;
     u32 lane, ekey; // HW lane; emulated-warp key within the HW warp (63: idle)
     u32 nlog;
+    u32 evm;        // kinds with a recorded event (bit k: PgCold::ecnt[k] / ebest[k] are valid)
+    u32 fl;         // PG_FAST: this thread saw a possible race / write-log overflow (instance re-run exactly)
     u32 l0cell, l0val, l0site;  // write-log entry 0 (registers; entries 1.. live in PgCold)
     u32 fuel;
     u32 sg;         // byte offset of this instance's shared region in pg_dsmem
@@ -135,9 +138,8 @@ struct PgCold {     // per-emulated-thread state that lives in local memory
     u32 lcell[PG_WMAX];   // write log entries 1.. (X3): cell id = array << 24 | flat
     u32 lval[PG_WMAX];
     u16 lsite[PG_WMAX];
-    u32 ecnt[PG_NK];      // events per kind
-    u32 ebest[PG_NK][8];  // minimum event per kind (X16)
-    u32 any;              // some event recorded
+    u32 ecnt[PG_NK];      // events per kind       (valid where PgT::evm has bit k: never initialised,
+    u32 ebest[PG_NK][8];  // minimum event per kind  so threads without events touch no local memory) (X16)
 };
 
 __device__ __forceinline__ bool pg_lex_less(const u32* a, const u32* b) {
@@ -148,16 +150,20 @@ __device__ __forceinline__ bool pg_lex_less(const u32* a, const u32* b) {
     return false;
 }
 
-__device__ __noinline__ void pg_event(PgCold& c, u32 kind, u32 round, u32 arr, u32 addr, u32 ta, u32 tb, u32 site,
-                                      u32 va, u32 vb) {
+// Records an event of `kind`; `evm` is the caller's event mask (PgT::evm).  Returns the
+// kind's bit, which the caller ORs into its mask.
+__device__ __noinline__ u32 pg_event(PgCold& c, u32 evm, u32 kind, u32 round, u32 arr, u32 addr, u32 ta, u32 tb,
+                                     u32 site, u32 va, u32 vb) {
     u32 e[8] = {round, arr, addr, ta, tb, site, va, vb};
-    if (c.ecnt[kind] == 0 || pg_lex_less(e, c.ebest[kind])) {
+    const u32 has = (evm >> kind) & 1u;
+    if (!has || pg_lex_less(e, c.ebest[kind])) {
 #pragma unroll
         for (int i = 0; i < 8; i++) c.ebest[kind][i] = e[i];
     }
-    c.ecnt[kind]++;
-    c.any = 1u;
+    c.ecnt[kind] = has ? c.ecnt[kind] + 1u : 1u;
+    return 1u << kind;
 }
+#define PG_EVENT(t, c, ...) ((t).evm |= pg_event((c), (t).evm, __VA_ARGS__))
 
 // stamps: step (20 bits, >= 1) and block-local tid (12 bits)
 __device__ __forceinline__ u32 pg_stamp_min(const PgC& C, const PgT& t) { return ((0xFFFFFu - C.step) << 12) | t.tlin; }
@@ -165,6 +171,25 @@ __device__ __forceinline__ u32 pg_stamp_max(const PgC& C, const PgT& t) { return
 __device__ __forceinline__ u32 pg_owner_step(u32 own) { return 0xFFFFFu - (own >> 12); }
 
 __device__ __forceinline__ u32* pg_sh(const PgT& t, u32 off) { return (u32*)(pg_dsmem + t.sg + off); }
+
+#ifndef PG_FAST
+#define PG_FAST 0
+#endif
+#if PG_FAST
+// Optimistic pass: stores commit in place and every round ends at one
+// barrier.  That equals the round semantics X3/X4 whenever no race occurs, so the pass
+// only has to DETECT that a race may have occurred; the instance is then re-run by the
+// exact protocol.  A second writer of a cell in a round sees the first one's owner stamp
+// in atomicMin's return value (WW).  Readers stamp the cell (reader stamps of the round's
+// parity set, step & 1); after the round's barrier every writer re-reads the reader
+// stamps of the cells it wrote - all reads of the round are visible then, whether they
+// came before or after the write - while the next round stamps the other set (RW).
+__shared__ u32 pg_sAbort;   // some thread of the CTA flagged (CTA-wide blocks)
+// reader stamps show a reader of round `step` other than this thread
+__device__ __forceinline__ u32 pg_fast_readers(u32 step, const PgT& t, u32 rmin, u32 rmax) {
+    return (rmax >> 12) == step && (((rmin & 0xFFFu) != t.tlin) | ((rmax & 0xFFFu) != t.tlin));
+}
+#endif
 
 // ------------------------------------------------------------------ bank / coalescing (X9, H6)
 __device__ __forceinline__ void pg_site_stat(u64* st, u32 space, u32 bad, u32 metric, u32 ideal, u32 lanes) {
@@ -180,8 +205,8 @@ __device__ __forceinline__ void pg_site_stat(u64* st, u32 space, u32 bad, u32 me
 
 // All 32 lanes of the warp call these together (the generated code keeps warps
 // converged around every access site).
-__device__ __noinline__ void pg_bank_shared(u32 round, u32 lane, u32 ekey0, u32 tlin, u32 gtid, PgCold& c, u64* sstats,
-                                            u32 active, u32 rec, u32 flat, u32 site) {
+__device__ __noinline__ u32 pg_bank_shared(u32 round, u32 lane, u32 ekey0, u32 tlin, u32 gtid, PgCold& c, u32 evm,
+                                           u64* sstats, u32 active, u32 rec, u32 flat, u32 site) {
     u32 ekey = ekey0;
     if (PG_BANK16) ekey = ekey * 2u + ((tlin >> 4) & 1u);
     const u32 seg = __match_any_sync(PG_FULL, ekey);
@@ -200,12 +225,13 @@ __device__ __noinline__ void pg_bank_shared(u32 round, u32 lane, u32 ekey0, u32 
     const u32 tb = __reduce_min_sync(seg, (active && bank == bstar && flat != astar) ? gtid : PG_NEVER);
     if (amask && lane == (u32)(__ffs(amask) - 1)) {
         if (sstats && site < PG_NSTATS) pg_site_stat(sstats + site * 8, 1, deg > 1, deg, 1, __popc(amask));
-        if (deg > 1) pg_event(c, PGK_BANK, round, rec, astar, ta, tb, site, deg, 0);
+        if (deg > 1) return pg_event(c, evm, PGK_BANK, round, rec, astar, ta, tb, site, deg, 0);
     }
+    return 0u;
 }
 
-__device__ __noinline__ void pg_coal_global(u32 round, u32 lane, u32 ekey, u32 gtid, PgCold& c, u64* sstats,
-                                            u32 active, u32 rec, u32 flat, u32 site) {
+__device__ __noinline__ u32 pg_coal_global(u32 round, u32 lane, u32 ekey, u32 gtid, PgCold& c, u32 evm,
+                                           u64* sstats, u32 active, u32 rec, u32 flat, u32 site) {
     const u32 seg = __match_any_sync(PG_FULL, ekey);
     const u32 amask = __ballot_sync(PG_FULL, active) & seg;
     const u32 w = active ? flat : 0u;
@@ -220,8 +246,9 @@ __device__ __noinline__ void pg_coal_global(u32 round, u32 lane, u32 ekey, u32 g
     const u32 tb = __reduce_max_sync(seg, active ? gtid : 0u);
     if (amask && lane == (u32)(__ffs(amask) - 1)) {
         if (sstats && site < PG_NSTATS) pg_site_stat(sstats + site * 8, 2, sectors > ideal, sectors, ideal, __popc(amask));
-        if (sectors > ideal) pg_event(c, PGK_UNCOAL, round, rec, amin, ta, tb, site, sectors, ideal);
+        if (sectors > ideal) return pg_event(c, evm, PGK_UNCOAL, round, rec, amin, ta, tb, site, sectors, ideal);
     }
+    return 0u;
 }
 
 // ------------------------------------------------------------------ loads / stores
@@ -239,23 +266,21 @@ __device__ __forceinline__ u32 pg_log_find(const PgT& t, const PgCold& c, u32 ce
     return 0u;
 }
 
-__device__ __noinline__ void pg_log_write_slow(u32 round, u32 gtid, u32& nlog, PgCold& c, u32 cell, u32 val, u32 site,
-                                               u32 rec, u32 flat) {
+// Returns the new log length, or PG_NEVER when the write-log limit dropped the write
+// (X19; the caller records the LIMIT event).
+__device__ __noinline__ u32 pg_log_write_slow(u32 nlog, PgCold& c, u32 cell, u32 val, u32 site) {
     for (u32 i = 1; i < nlog; i++) {
         if (c.lcell[i] == cell) {
             c.lval[i] = val;
             c.lsite[i] = (u16)site;
-            return;
+            return nlog;
         }
     }
-    if (nlog >= PG_WMAX) {  // X19: write-log limit, the write is dropped
-        pg_event(c, PGK_LIMIT, round, rec, flat, gtid, PG_NEVER, site, 1, 0);
-        return;
-    }
+    if (nlog >= PG_WMAX) return PG_NEVER;
     c.lcell[nlog] = cell;
     c.lval[nlog] = val;
     c.lsite[nlog] = (u16)site;
-    nlog++;
+    return nlog + 1u;
 }
 
 __device__ __forceinline__ void pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell, u32 val, u32 site, u32 rec,
@@ -269,7 +294,9 @@ __device__ __forceinline__ void pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell
         t.l0val = val;
         t.l0site = site;
     } else {
-        pg_log_write_slow(C.round, t.gtid, t.nlog, c, cell, val, site, rec, flat);
+        const u32 n = pg_log_write_slow(t.nlog, c, cell, val, site);
+        if (n == PG_NEVER) PG_EVENT(t, c, PGK_LIMIT, C.round, rec, flat, t.gtid, PG_NEVER, site, 1, 0);
+        else t.nlog = n;
     }
 }
 
@@ -312,16 +339,24 @@ template <int A, bool RD, bool LOG>
 __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site) {
     const u32 inb = flat < PG_SH(A, size);
 #if PG_BANKCHK
-    pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
+    t.evm |= pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, t.evm, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
 #endif
     if (!pe) return 0u;
     if (!inb) {
         const u32 pv = pg_poison_sh(t, PG_ARR(A).rec_id, flat);
 #if PG_OOBCHK
-        pg_event(c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
+        PG_EVENT(t, c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
 #endif
         return pv;
     }
+#if PG_FAST
+    if (RD && PG_T > 1u) {
+        const u32 so = (C.step & 1u) * PG_SH(A, size) + flat;
+        atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + so, pg_stamp_min(C, t));
+        atomicMax(pg_sh(t, PG_SH(A, s_rmax)) + so, pg_stamp_max(C, t));
+    }
+    const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
+#else
 #if PG_RACECHK
     if (RD && PG_T > 1u) {
         atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + flat, pg_stamp_min(C, t));
@@ -336,10 +371,11 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
         return v;
     }
     const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
+#endif
     if (pg_owner_step(own) < C.step0) {  // never written in this block (X6)
         const u32 pv = pg_poison_sh(t, PG_ARR(A).rec_id, flat);
 #if PG_OOBCHK
-        pg_event(c, PGK_UNINIT, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
+        PG_EVENT(t, c, PGK_UNINIT, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
 #endif
 #if PG_DATAFLOW
         pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER);
@@ -353,20 +389,77 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
     return pg_sh(t, PG_SH(A, s_val))[flat];
 }
 
+#if PG_FAST
+// write log of the optimistic pass: cells whose readers are checked after the barrier
+// (low 16 bits: logged cells; high 16 bits: stores this round, X19's W_max)
+__device__ __forceinline__ void pg_flog(PgT& t, PgCold& c, u32 cell) {
+    const u32 n = t.nlog & 0xFFFFu;
+    if (n == 0u) {
+        t.l0cell = cell;
+        t.nlog += 1u;
+    } else if (t.l0cell != cell) {
+        const u32 m = pg_log_write_slow(n, c, cell, 0u, 0u);
+        if (m == PG_NEVER) t.fl = 1u;
+        else t.nlog += m - n;
+    }
+}
+__device__ __forceinline__ void pg_fcount(PgT& t) {
+    t.nlog += 0x10000u;
+    t.fl |= (t.nlog >> 16) > (u32)PG_WMAX;   // more stores than the write log holds: LIMIT is decided exactly
+}
+// in-place commit (optimistic pass): owner stamp (WW detection), value, reader check log
+template <int A, bool RDA>
+__device__ __forceinline__ void pg_commit_sh(const PgC& C, PgT& t, PgCold& c, u32 flat, u32 val) {
+    u32* own = pg_sh(t, PG_SH(A, s_own)) + flat;
+    const u32 me = pg_stamp_min(C, t);
+    if (PG_T > 1u) {
+        const u32 old = atomicMin(own, me);
+        t.fl |= (old != me) & ((old >> 12) == (me >> 12));   // a second writer this round (WW)
+        if (RDA) pg_flog(t, c, ((u32)A << 24) | flat);
+    } else {
+        *own = me;
+    }
+    pg_sh(t, PG_SH(A, s_val))[flat] = val;
+    pg_fcount(t);
+}
+// after the round's barrier: readers of a cell this thread wrote in round `step`
 template <int A>
+__device__ __forceinline__ void pg_fcheck_sh(u32 step, PgT& t, u32 flat) {
+    const u32 so = (step & 1u) * PG_SH(A, size) + flat;
+    t.fl |= pg_fast_readers(step, t, pg_sh(t, PG_SH(A, s_rmin))[so], pg_sh(t, PG_SH(A, s_rmax))[so]);
+}
+template <int A>
+__device__ __forceinline__ void pg_fcheck_gt(u32 step, PgT& t, u32 flat) {
+    const u64 so = (u64)(step & 1u) * PG_ARR(A).size + flat;
+    t.fl |= pg_fast_readers(step, t, t.arena[PG_ARR(A).off_rmin + so], t.arena[PG_ARR(A).off_rmax + so]);
+}
+template <class K>
+__device__ __forceinline__ void pg_fcheck_all(u32 step, PgT& t, PgCold& c) {
+    const u32 n = t.nlog & 0xFFFFu;
+    if (n == 0u) return;
+    K::fcheck_one(step, t, t.l0cell);
+    for (u32 i = 1; i < n; i++) K::fcheck_one(step, t, c.lcell[i]);
+}
+#endif
+
+template <int A, bool RDA = false>
 __device__ __forceinline__ void pg_st_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 val, u32 site) {
     const u32 inb = flat < PG_SH(A, size);
 #if PG_BANKCHK
-    pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
+    t.evm |= pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, t.evm, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
 #endif
     if (!pe) return;
     if (!inb) {
 #if PG_OOBCHK
-        pg_event(c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, val, 1);
+        PG_EVENT(t, c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, val, 1);
 #endif
         return;
     }
+#if PG_FAST
+    pg_commit_sh<A, RDA>(C, t, c, flat, val);
+#else
     pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+#endif
 }
 
 // XB bookkeeping (X4): first and last block that accessed a global cell.  Kept
@@ -385,17 +478,25 @@ template <int A, bool RD, bool LOG>
 __device__ __forceinline__ u32 pg_ld_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site) {
     const u32 inb = flat < PG_ARR(A).size;
 #if PG_COALCHK
-    pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
+    t.evm |= pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, t.evm, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
 #endif
     if (!pe) return 0u;
     if (!inb) {
         const u32 pv = pg_m(pg_rand32(t.seed, PG_ARR(A).gid, flat));
 #if PG_OOBCHK
-        pg_event(c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
+        PG_EVENT(t, c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
 #endif
         return pv;
     }
     pg_xb_mark<A>(t, flat);
+#if PG_FAST
+    if (RD && PG_T > 1u) {
+        const u64 so = (u64)(C.step & 1u) * PG_ARR(A).size + flat;
+        atomicMin(t.arena + PG_ARR(A).off_rmin + so, pg_stamp_min(C, t));
+        atomicMax(t.arena + PG_ARR(A).off_rmax + so, pg_stamp_max(C, t));
+    }
+    return t.arena[PG_ARR(A).off_val + flat];
+#else
 #if PG_RACECHK
     if (RD && PG_T > 1u) {
         atomicMin(t.arena + PG_ARR(A).off_rmin + flat, pg_stamp_min(C, t));
@@ -414,23 +515,41 @@ __device__ __forceinline__ u32 pg_ld_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
                  t.arena[PG_ARR(A).off_own + flat], pg_sL.off_step0);
 #endif
     return t.arena[PG_ARR(A).off_val + flat];
+#endif
 }
 
-template <int A>
+template <int A, bool RDA = false>
 __device__ __forceinline__ void pg_st_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 val, u32 site) {
     const u32 inb = flat < PG_ARR(A).size;
 #if PG_COALCHK
-    pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
+    t.evm |= pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, t.evm, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
 #endif
     if (!pe) return;
     if (!inb) {
 #if PG_OOBCHK
-        pg_event(c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, val, 1);
+        PG_EVENT(t, c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, val, 1);
 #endif
         return;
     }
     pg_xb_mark<A>(t, flat);
+#if PG_FAST
+    {
+        u32* own = t.arena + PG_ARR(A).off_own + flat;
+        const u32 me = pg_stamp_min(C, t);
+        if (PG_T > 1u) {
+            const u32 old = atomicMin(own, me);
+            t.fl |= (old != me) & ((old >> 12) == (me >> 12));
+            if (RDA) pg_flog(t, c, ((u32)A << 24) | flat);
+        } else {
+            *own = me;
+        }
+        t.arena[PG_ARR(A).off_val + flat] = val;
+        t.arena[PG_ARR(A).off_lw + flat] = t.gtid + 1u;
+        pg_fcount(t);
+    }
+#else
     pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+#endif
 }
 
 // Global array this kernel only reads: the instance's input region.
@@ -438,13 +557,13 @@ template <int A>
 __device__ __forceinline__ u32 pg_ld_gi(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site) {
     const u32 inb = flat < PG_ARR(A).size;
 #if PG_COALCHK
-    pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
+    t.evm |= pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, t.evm, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
 #endif
     if (!pe) return 0u;
     if (!inb) {
         const u32 pv = pg_m(pg_rand32(t.seed, PG_ARR(A).gid, flat));
 #if PG_OOBCHK
-        pg_event(c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
+        PG_EVENT(t, c, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
 #endif
         return pv;
     }
@@ -460,7 +579,7 @@ __device__ __forceinline__ u32 pg_priv_ok(PgC& C, PgT& t, PgCold& c, u32 pe, u32
     if (!pe) return 0u;
     if (flat < size) return 1u;
 #if PG_OOBCHK
-    pg_event(c, PGK_OOB, C.round, rec, flat, t.gtid, PG_NEVER, site, is_store ? val : 0u, is_store);
+    PG_EVENT(t, c, PGK_OOB, C.round, rec, flat, t.gtid, PG_NEVER, site, is_store ? val : 0u, is_store);
 #endif
     return 0u;
 }
@@ -468,7 +587,7 @@ __device__ __forceinline__ u32 pg_priv_ok(PgC& C, PgT& t, PgCold& c, u32 pe, u32
 // ------------------------------------------------------------------ loops (fuel, X19)
 __device__ __forceinline__ void pg_tick(PgC& C, PgT& t, PgCold& c, u32 act) {
     if (act && ++t.fuel > C.fuel) {
-        pg_event(c, PGK_LIMIT, C.round, PG_NEVER, 0, t.gtid, PG_NEVER, PG_NEVER, 2, 0);
+        PG_EVENT(t, c, PGK_LIMIT, C.round, PG_NEVER, 0, t.gtid, PG_NEVER, PG_NEVER, 2, 0);
         t.live = 0;
     }
 }
@@ -493,11 +612,12 @@ __device__ __forceinline__ void pg_claim_gt(const PgC& C, const PgT& t, u32 flat
 #endif
 }
 
-__device__ __noinline__ void pg_race_check(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 val, u32 site,
-                                           u32 rec, u32 flat, u32 own, u32 wmax, u32 has_readers, u32 rmin, u32 rmax) {
+__device__ __noinline__ u32 pg_race_check(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 evm, u32 val,
+                                          u32 site, u32 rec, u32 flat, u32 own, u32 wmax, u32 has_readers, u32 rmin,
+                                          u32 rmax) {
     const u32 base = gtid - tlin;
     const u32 w0 = own & 0xFFFu, w1 = wmax & 0xFFFu;
-    if (w1 != w0 && tlin == w0) pg_event(c, PGK_WW, round, rec, flat, gtid, base + w1, site, val, 0);
+    if (w1 != w0 && tlin == w0) evm |= pg_event(c, evm, PGK_WW, round, rec, flat, gtid, base + w1, site, val, 0);
     if (has_readers && (rmax >> 12) == step) {
         const u32 r0 = rmin & 0xFFFu, r1 = rmax & 0xFFFu;
         if (!(r0 == r1 && w0 == w1 && r0 == w0)) {
@@ -505,13 +625,14 @@ __device__ __noinline__ void pg_race_check(u32 round, u32 step, u32 tlin, u32 gt
             if (r0 != w0) { ta = w0; tb = r0; }
             else if (r1 != w0) { ta = w0; tb = r1; }
             else { ta = w1; tb = r0; }
-            if (tlin == ta) pg_event(c, PGK_RW, round, rec, flat, base + ta, base + tb, site, val, 0);
+            if (tlin == ta) evm |= pg_event(c, evm, PGK_RW, round, rec, flat, base + ta, base + tb, site, val, 0);
         }
     }
+    return evm;
 }
 
 template <int A, bool RD>
-__device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
+__device__ __forceinline__ void pg_check_sh(const PgC& C, PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
     if (PG_T == 1u) {
         pg_sh(t, PG_SH(A, s_own))[flat] = pg_stamp_min(C, t);
         pg_sh(t, PG_SH(A, s_val))[flat] = val;
@@ -527,14 +648,14 @@ __device__ __forceinline__ void pg_check_sh(const PgC& C, const PgT& t, PgCold& 
         // (a cell only its writer read this round is no RW race: skip the slow path)
         if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
             (RD && (rmax >> 12) == C.step && (((rmin ^ own) | (rmax ^ own)) & 0xFFFu)))
-            pg_race_check(C.round, C.step, t.tlin, t.gtid, c, val, site, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin,
-                          rmax);
+            t.evm = pg_race_check(C.round, C.step, t.tlin, t.gtid, c, t.evm, val, site, PG_ARR(A).rec_id, flat, own,
+                                  wmax, RD, rmin, rmax);
     }
 #endif
 }
 
 template <int A, bool RD>
-__device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
+__device__ __forceinline__ void pg_check_gt(const PgC& C, PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
     if (PG_T == 1u) {
         t.arena[PG_ARR(A).off_own + flat] = pg_stamp_min(C, t);
         t.arena[PG_ARR(A).off_val + flat] = val;
@@ -554,8 +675,8 @@ __device__ __forceinline__ void pg_check_gt(const PgC& C, const PgT& t, PgCold& 
         // (a cell only its writer read this round is no RW race: skip the slow path)
         if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
             (RD && (rmax >> 12) == C.step && (((rmin ^ own) | (rmax ^ own)) & 0xFFFu)))
-            pg_race_check(C.round, C.step, t.tlin, t.gtid, c, val, site, PG_ARR(A).rec_id, flat, own, wmax, RD, rmin,
-                          rmax);
+            t.evm = pg_race_check(C.round, C.step, t.tlin, t.gtid, c, t.evm, val, site, PG_ARR(A).rec_id, flat, own,
+                                  wmax, RD, rmin, rmax);
     }
 #endif
 }
@@ -569,7 +690,7 @@ __device__ __forceinline__ void pg_claim_all(const PgC& C, const PgT& t, const P
     for (u32 i = 1; i < t.nlog; i++) K::claim_one(C, t, c.lcell[i]);
 }
 template <class K>
-__device__ __forceinline__ void pg_check_all(const PgC& C, const PgT& t, PgCold& c) {
+__device__ __forceinline__ void pg_check_all(const PgC& C, PgT& t, PgCold& c) {
     if (t.nlog == 0u) return;
     K::check_one(C, t, c, t.l0cell, t.l0val, t.l0site);
     for (u32 i = 1; i < t.nlog; i++) K::check_one(C, t, c, c.lcell[i], c.lval[i], c.lsite[i]);
@@ -601,6 +722,39 @@ __device__ __noinline__ void pg_snapshot(const PgC& C, const PgT& t) {
 template <class K, bool LAST>
 __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& alive_rounds) {
     const bool warp_blocks = PG_T <= 32u;
+#if PG_FAST
+    // stores committed in place: one barrier (with the early-exit vote) ends the round;
+    // once some thread flagged a race the item stops (every instance of the warp / CTA is
+    // re-run exactly, so finishing it would be wasted work)
+    C.round++;
+    if (warp_blocks) __syncwarp();
+    if (LAST) {
+        if (!warp_blocks) __syncthreads();
+        pg_fcheck_all<K>(C.step, t, c);
+        return false;
+    }
+    int more;
+    if (warp_blocks) {
+        more = __any_sync(PG_FULL, t.live);
+        C.abort = __any_sync(PG_FULL, t.fl);
+    } else {
+        if (t.fl) pg_sAbort = 1u;
+        more = __syncthreads_or((int)t.live);
+        C.abort = pg_sAbort;
+    }
+    if (C.abort) {
+        t.fl = 1u;
+        return false;
+    }
+    pg_fcheck_all<K>(C.step, t, c);   // (flags found here stop the item at the next round end)
+    if (!more) return false;
+    C.step++;
+    C.ufuel = 0;
+    t.nlog = 0;
+    t.fuel = 0;
+    alive_rounds += t.live;
+    return true;
+#else
     if (warp_blocks) __syncwarp(); else __syncthreads();
     pg_claim_all<K>(C, t, c);
     if (warp_blocks) __syncwarp(); else __syncthreads();
@@ -619,6 +773,7 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
     t.fuel = 0;
     alive_rounds += t.live;
     return true;
+#endif
 }
 
 // ------------------------------------------------------------------ records (H8)
@@ -669,20 +824,24 @@ __device__ __noinline__ void pg_slot_update(PgSlot* s, u32 cnt, const u32* best)
     atomicExch(&s->lock, 0u);
 }
 
-__device__ __noinline__ void pg_flush_cta(const PgParams& P, u32 lane, u32 warp, PgCold& c, u32 valid, u64 slot0,
-                                          PgFlushEntry* sh /* [32] in shared memory */) {
+__device__ __noinline__ void pg_flush_cta(const PgParams& P, u32 lane, u32 warp, PgCold& c, u32 evm, u32 valid,
+                                          u64 slot0, PgFlushEntry* sh /* [32] in shared memory */) {
     const u32 nwarps = blockDim.x >> 5;
+    const u32 warp_evm = __reduce_or_sync(PG_FULL, valid ? evm : 0u);
     for (u32 k = 0; k < PG_NK; k++) {
-        if (!__syncthreads_or((int)(valid && c.ecnt[k] != 0u))) continue;
+        if (!__syncthreads_or((int)((warp_evm >> k) & 1u))) continue;
         if (lane == 0) sh[warp].slot = ~0ull;
         __syncwarp();
-        u32 pending = valid && c.ecnt[k] != 0u;
+        u32 pending = valid && ((evm >> k) & 1u);
         bool first = true;
         for (;;) {
             if (!__any_sync(PG_FULL, pending)) break;
             u32 leader, cnt, members, best[8];
             u64 key;
-            pg_warp_merge(pending, slot0, c.ecnt[k], c.ebest[k], lane, leader, key, cnt, best, members);
+            u32 f_in[8];
+#pragma unroll
+            for (int i = 0; i < 8; i++) f_in[i] = pending ? c.ebest[k][i] : PG_NEVER;
+            pg_warp_merge(pending, slot0, pending ? c.ecnt[k] : 0u, f_in, lane, leader, key, cnt, best, members);
             if (lane == leader) {
                 if (first) {   // the common case: one instance per warp -> deposit for the CTA merge
                     sh[warp].slot = key;
@@ -743,6 +902,18 @@ __device__ __forceinline__ u32 pg_init_value(const PgParams& P, u64 seed, u32 gi
 template <class K>
 __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     __shared__ u32 s_flag;
+    if (P.seq) {
+        // re-runs: only items with a flagged instance (seq 1: a global cell shared between
+        // blocks; seq 2: a race the optimistic pass flagged)
+        if (threadIdx.x == 0) {
+            const PgWork& w = P.work[wi];
+            u32 f = 0;
+            for (u32 i = 0; i < w.nseeds; i++) f |= P.xb_flag[w.inst0 + i];
+            s_flag = f;
+        }
+        __syncthreads();
+        if (!s_flag) return;
+    }
     {
         const u32* src = (const u32*)&P.launches[P.work[wi].launch];
         u32* dst = (u32*)&pg_sL;
@@ -756,15 +927,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 #endif
     __syncthreads();
     const u32 G = pg_sW.ngroups, GB = pg_sW.gb;
-    if (P.seq) {
-        // re-run only seed groups in which some instance shared a global cell between blocks
-        if (threadIdx.x == 0) {
-            u32 f = 0;
-            for (u32 i = 0; i < pg_sW.nseeds; i++) f |= P.xb_flag[pg_sW.inst0 + i];
-            s_flag = f;
-        }
-        __syncthreads();
-        if (!s_flag) return;
+    if (P.seq == 1u) {
         // fresh arenas and slots for every seed of the group (the parallel pass is discarded)
         for (u32 ms = 0; ms < pg_sW.nseeds; ms++) {
             const u64 seed = P.seed_base + (u64)(pg_sW.seed_j0 + ms * pg_sW.seed_jstep);
@@ -777,8 +940,10 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                     ar[R.off_own + i] = PG_NEVER;
                     ar[R.off_lw + i] = 0u;
                     if (R.off_wmax != ~0ull) ar[R.off_wmax + i] = 0u;
-                    if (R.off_rmin != ~0ull) ar[R.off_rmin + i] = PG_NEVER;
-                    if (R.off_rmax != ~0ull) ar[R.off_rmax + i] = 0u;
+                    for (u32 q = 0; q < R.rsets; q++) {
+                        if (R.off_rmin != ~0ull) ar[R.off_rmin + (u64)q * R.size + i] = PG_NEVER;
+                        if (R.off_rmax != ~0ull) ar[R.off_rmax + (u64)q * R.size + i] = 0u;
+                    }
                     if (R.off_xf != ~0ull) { ar[R.off_xf + i] = PG_NEVER; ar[R.off_xl + i] = 0u; }
                 }
             }
@@ -788,6 +953,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 sl->has = 0;
                 sl->lock = 0;
             }
+            if (threadIdx.x == 0u) P.inst_cnt[pg_sW.inst0 + ms] = 0ull;   // counted again below
         }
         __threadfence();
         __syncthreads();
@@ -817,6 +983,10 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 
     PgC C;
     C.step = 0;
+    C.abort = 0;
+#if PG_FAST
+    if (threadIdx.x == 0) pg_sAbort = 0u;   // (published by the barrier below)
+#endif
     C.fuel = P.fuel;
     const u32 lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
     u32 g, tl0, lane_ok, ekey;
@@ -832,7 +1002,8 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         lane_ok = 1u;
         ekey = 0u;
     }
-    const u32 inst_ok = lane_ok && g < G;
+    // (exact re-run, P.seq == 2: only the instances the optimistic pass flagged)
+    const u32 inst_ok = lane_ok && g < G && (P.seq != 2u || P.xb_flag[pg_sW.inst0 + g / GB] != 0u);
     const u32 gc = inst_ok ? g : 0u;
     const u32 ms = gc / GB, bs = gc % GB;
     typename K::Frame F[PG_VMAX];
@@ -855,11 +1026,10 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         t.input = P.input + pg_sW.input_off + (u64)ms * pg_sL.input_stride;
         t.sg = gc * gbytes;
         t.l0cell = t.l0val = t.l0site = 0u;
-        for (u32 k = 0; k < PG_NK; k++) Cd[v].ecnt[k] = 0;
-        Cd[v].any = 0u;
+        t.evm = 0u;
+        t.fl = 0u;
         t.live = ok;
     }
-    __shared__ u64 s_part[32];   // per-warp instance counts
     __syncthreads();
     const bool grid_1d = pg_sL.gdim[1] == 1u && pg_sL.gdim[2] == 1u;
     const bool grid_pow2 = !(pg_sL.gdim[0] & (pg_sL.gdim[0] - 1u)) && !(pg_sL.gdim[1] & (pg_sL.gdim[1] - 1u));
@@ -922,6 +1092,15 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 r = K::seg(F[v], C, T[v], Cd[v], sstats, resume);
             }
             alive_rounds += any_start;
+            u32 any = 0;
+#if PG_FAST
+            if (warp_blocks) __syncwarp();
+#pragma unroll
+            for (u32 v = 0; v < PG_VMAX; v++) {
+                if (v >= V) break;
+                any |= T[v].live;
+            }
+#else
             if (warp_blocks) __syncwarp(); else __syncthreads();
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
@@ -929,15 +1108,43 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 pg_claim_all<K>(C, T[v], Cd[v]);
             }
             if (warp_blocks) __syncwarp(); else __syncthreads();
-            u32 any = 0;
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
                 pg_check_all<K>(C, T[v], Cd[v]);
                 any |= T[v].live;
             }
+#endif
             C.round++;
+#if PG_FAST
+            u32 fl = 0;
+#pragma unroll
+            for (u32 v = 0; v < PG_VMAX; v++) {
+                if (v >= V) break;
+                fl |= T[v].fl;
+            }
+            int more;
+            if (warp_blocks) {
+                more = __any_sync(PG_FULL, any);
+                C.abort = __any_sync(PG_FULL, fl);
+            } else {
+                if (fl) pg_sAbort = 1u;
+                more = __syncthreads_or((int)any);
+                C.abort = pg_sAbort;
+            }
+            if (C.abort) {
+#pragma unroll
+                for (u32 v = 0; v < PG_VMAX; v++) T[v].fl = 1u;
+                break;
+            }
+#pragma unroll
+            for (u32 v = 0; v < PG_VMAX; v++) {
+                if (v >= V) break;
+                pg_fcheck_all<K>(C.step, T[v], Cd[v]);
+            }
+#else
             const int more = warp_blocks ? __any_sync(PG_FULL, any) : __syncthreads_or((int)any);
+#endif
             if (r == PG_END || !more) break;
             resume = r;
         }
@@ -965,12 +1172,13 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             if (inst_ok && tl0 == 0u) s_grounds[g] = 0u;
         }
         inst += (u64)T_ * grounds;
+        if (C.abort) break;   // (PG_FAST; warp- or CTA-uniform like the barriers above)
     }
     __syncthreads();
 #if PG_RACECHK
     // X4: cross-block races on global cells written by this kernel (sequential pass: the
     // CTA owns whole instances; the parallel pass leaves them to the flagged re-run)
-    if (P.seq && pg_sL.nblocks > 1) {
+    if (P.seq == 1u && pg_sL.nblocks > 1) {
 #pragma unroll
         for (u32 v = 0; v < PG_VMAX; v++) {
             if (v >= V) break;
@@ -985,7 +1193,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 const u32* val = t.arena + ar.off_val;
                 for (u32 i = t.tlin; i < ar.size; i += T_)
                     if (lw[i] && xf[i] != xl[i])
-                        pg_event(Cd[v], PGK_XB, 0xFFFFu, ar.rec_id, i, xf[i] - 1u, xl[i] - 1u, PG_NEVER, val[i], 0u);
+                        PG_EVENT(t, Cd[v], PGK_XB, 0xFFFFu, ar.rec_id, i, xf[i] - 1u, xl[i] - 1u, PG_NEVER, val[i], 0u);
             }
         }
     }
@@ -996,34 +1204,46 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 #pragma unroll
         for (u32 v = 0; v < PG_VMAX; v++) {
             if (v >= V) break;
-            any_ev |= Cd[v].any;
+            any_ev |= T[v].evm;
         }
         if (__syncthreads_or((int)any_ev)) {
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
-                pg_flush_cta(P, lane, warp, Cd[v], inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)ms * pg_sW.slot_step,
+                pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)ms * pg_sW.slot_step,
                              s_flush);
             }
         }
     }
-    // instances (X19): warp sums, then one global atomic per CTA
+#if PG_FAST
+    {   // flag instances with a possible race for the exact re-run
+        u32 fl = 0;
+#pragma unroll
+        for (u32 v = 0; v < PG_VMAX; v++) {
+            if (v >= V) break;
+            fl |= T[v].fl;
+        }
+        if (fl && inst_ok) P.xb_flag[pg_sW.inst0 + ms] = 1u;
+    }
+#endif
+    // instances (X19) per batch-local instance (a re-run replaces its instance's count):
+    // one atomic per warp when the warp's groups belong to one instance (block-major packing)
     if (P.count_inst) {
         u64 x = (inst_ok && tl0 == 0u) ? inst : 0ull;
+        const u32 key = x ? pg_sW.inst0 + ms : PG_NEVER;
+        const u32 k0 = __reduce_min_sync(PG_FULL, key);
+        if (__all_sync(PG_FULL, key == PG_NEVER || key == k0)) {
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(PG_FULL, x, o);
-        if (lane == 0u) s_part[warp] = x;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            u64 sum = 0;
-            for (u32 w = 0; w < (blockDim.x + 31u) / 32u; w++) sum += s_part[w];
-            if (sum) atomicAdd(&P.counts[0], sum);
+            for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(PG_FULL, x, o);
+            if (lane == 0u && x) atomicAdd(&P.inst_cnt[k0], x);
+        } else if (x) {
+            atomicAdd(&P.inst_cnt[key], x);
         }
     }
 #if PG_BANKCHK || PG_COALCHK
     __syncthreads();
     if (P.site_stats) {
-        u64* dst = P.site_stats + (u64)(P.seq ? pg_sW.launch : pg_sW.item) * P.max_sites * 8u;
+        u64* dst = P.site_stats + (u64)(P.seq == 1u ? pg_sW.launch : pg_sW.item) * P.max_sites * 8u;
         for (u32 i = threadIdx.x; i < PG_NSTATS * 8 && i < P.max_sites * 8; i += blockDim.x) {
             const u32 col = i & 7u;
             if (col == 3) atomicMax(&dst[i], sstats[i]);
@@ -1039,7 +1259,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 template <class K>
 __device__ __forceinline__ void pg_main(const PgParams& P) {
     const bool listed = P.work_count != nullptr;
-    const u32 n = listed ? *P.work_count : blockIdx.x + 1u;
+    const u32 n = listed ? *P.work_count : P.n_work ? P.n_work : blockIdx.x + 1u;
     for (u32 i = blockIdx.x; i < n; i += gridDim.x) {   // (one call site: one inlined copy)
         pg_item<K>(P, listed ? P.work_list[i] : i);
         __syncthreads();

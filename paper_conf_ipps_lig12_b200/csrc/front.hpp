@@ -125,6 +125,7 @@ struct CodegenOptions {
     uint32_t checks = 0;
     uint32_t bank_model = 0;
     uint32_t wmax = 32;
+    bool fast = false;   // optimistic pass: in-place commits, race detection only
 };
 std::string generate_cuda(const Kernel& k, const CodegenOptions& opt);
 

@@ -21,11 +21,16 @@ __device__ __forceinline__ u32 init_value(u32 mode, u32 range, u32 mask, u64 see
 
 // K1: blockIdx.y = job, blockIdx.x strides over the job's instances, threads
 // stride over the words.
+// With `flags`, only the jobs of region `only_target` and only flagged instances are
+// (re-)initialised: the exact re-run of the instances the optimistic pass flagged.
 __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ jobs, u32* arena_s, u32* arena_t,
-                                                     u32* input, u64 seed_base, u32 mode, u32 range, u32 mask) {
+                                                     u32* input, u64 seed_base, u32 mode, u32 range, u32 mask,
+                                                     const u32* flags, u32 only_target) {
     const PgFill f = jobs[blockIdx.y];
+    if (flags && f.target != only_target) return;
     u32* region = f.target == 0 ? arena_s : f.target == 1 ? arena_t : input;
     for (u32 inst = blockIdx.x; inst < f.n_inst; inst += gridDim.x) {
+        if (flags && !flags[f.inst0 + inst]) continue;
         u32* base = region + f.dst + (u64)inst * f.stride;
         const u64 seed = seed_base + (u64)f.j0 + (u64)inst * f.jstep;
         if (f.op == PGF_CONST) {
@@ -310,18 +315,63 @@ __global__ void __launch_bounds__(256) pg_compact(const PgSlot* __restrict__ slo
     }
 }
 
+// Before the exact re-run of flagged instances: clear their record slots (this kernel)
+// and their instance counts.
+__global__ void __launch_bounds__(256) pg_reset_flagged(const u32* flags, u32 n_inst, const u64* inst_slot0,
+                                                        u32 kernel, PgSlot* slots, u64* inst_cnt) {
+    const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n_inst || !flags[i]) return;
+    inst_cnt[i] = 0ull;
+    PgSlot* s = slots + inst_slot0[i] + (u64)kernel * PG_NK;
+    for (u32 k = 0; k < PG_NK; k++) {
+        s[k].count = 0ull;
+        s[k].lock = 0u;
+        s[k].has = 0u;
+    }
+}
+
+// X19: the batch's per-instance counts into the run's instance counter.
+__global__ void __launch_bounds__(1024) pg_count_reduce(const u64* inst_cnt, u32 n, unsigned long long* counts) {
+    u64 x = 0;
+    for (u32 i = threadIdx.x; i < n; i += blockDim.x) x += inst_cnt[i];
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(0xffffffffu, x, o);
+    __shared__ u64 part[32];
+    if ((threadIdx.x & 31u) == 0u) part[threadIdx.x >> 5] = x;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        u64 t = 0;
+        for (u32 w = 0; w < (blockDim.x + 31u) / 32u; w++) t += part[w];
+        atomicAdd(counts, t);
+    }
+}
+
 }  // namespace
 
 // ------------------------------------------------------------------ host wrappers (C++ linkage, used by api.cpp)
 namespace pgk {
 
 cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 max_inst, u32* arena_s, u32* arena_t, u32* input,
-                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st) {
+                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags,
+                       u32 only_target) {
     for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
         const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
         dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
-        pg_gen_inputs<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, seed_base, mode, range, mask);
+        pg_gen_inputs<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, seed_base, mode, range, mask, flags,
+                                            only_target);
     }
+    return cudaGetLastError();
+}
+
+cudaError_t reset_flagged(const u32* flags, u32 n_inst, const u64* inst_slot0, u32 kernel, PgSlot* slots,
+                          u64* inst_cnt, cudaStream_t st) {
+    if (!n_inst) return cudaSuccess;
+    pg_reset_flagged<<<(n_inst + 255) / 256, 256, 0, st>>>(flags, n_inst, inst_slot0, kernel, slots, inst_cnt);
+    return cudaGetLastError();
+}
+
+cudaError_t count_reduce(const u64* inst_cnt, u32 n, long long* counts, cudaStream_t st) {
+    if (!n) return cudaSuccess;
+    pg_count_reduce<<<1, 1024, 0, st>>>(inst_cnt, n, (unsigned long long*)counts);
     return cudaGetLastError();
 }
 

@@ -30,7 +30,8 @@ struct PgArr {
     u32 flags;      // bit0: reader stamps present (array read and written, race checks on)
     // shared arrays: byte offsets in the group's shared region
     u32 s_val, s_own, s_wmax, s_rmin, s_rmax;
-    u32 pad;
+    u32 rsets;      // reader-stamp sets (rmin/rmax hold rsets x size words): 2 when the optimistic
+                    // pass checks a round's readers after the next barrier (set = step & 1)
     // global arrays written by the kernel: u32-word offsets in the instance arena
     u64 off_val;    // values
     u64 off_own;    // owner stamp of the last commit: ((2^20-1 - step) << 12) | tid
@@ -89,15 +90,19 @@ struct PgParams {
     u32 max_sites;
     u32 kernel_idx;
     u32 fuel;
-    u32 seq;           // 0: block-parallel pass; 1: sequential re-run of flagged seed groups
+    u32 seq;           // 0: block-parallel pass; 1: sequential re-run of flagged seed groups;
+                       // 2: block-parallel exact re-run of the instances the optimistic pass flagged
     u32 input_mode, input_range, mask;
-    u32 count_inst;    // this pass counts instances (X19)
+    u32 count_inst;    // this pass counts instances (X19) into inst_cnt
+    u64* inst_cnt;     // per batch-local instance: instances counted (X19), summed by pg_count_reduce
     u32* df_rows;      // data-flow rows (12 words each), PG_CHK_DATAFLOW only
     u32* df_count;
     u32 df_cap;
     u32 pad2;
     const u32* work_list;   // sequential pass: indices (into work) of the items to run
-    const u32* work_count;  // their number (device); nullptr: one item per CTA
+    const u32* work_count;  // their number (device); nullptr: one item per CTA, or
+    u32 n_work;             // (non-zero) a grid-stride loop over this many items (exact re-run)
+    u32 pad3;
 };
 
 // K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive
@@ -113,6 +118,8 @@ struct PgFill {
     u32 gid;      // PRF tag (X8)
     u32 value;    // PGF_CONST fill value
     u32 target;   // 0 arena (src), 1 arena (tgt), 2 input region
+    u32 inst0;    // batch-local index of instance 0 (re-initialisation of flagged instances)
+    u32 pad;
 };
 
 // K2b (pg_xb_detect) job: one global array written by a kernel, for n_inst

@@ -71,8 +71,9 @@ SUBJECTS = sorted(f[:-4] for f in os.listdir(os.path.join(ROOT, "subjects")) if 
 def test_subject_compiles_for_sm100a(pgvc, name):
     from paper_conf_ipps_lig12_b200 import workloads as W
     ir = pgvc.load_ir(W.subject(name))
+    fast = 1 << 30   # internal bit: the optimistic pass
     for checks, bits in ((pgvc.CHK_RACE | pgvc.CHK_OOB, 32), (0, 32), (pgvc.CHK_BANK | pgvc.CHK_COALESCE, 32),
-                         (pgvc.CHK_RACE | pgvc.CHK_OOB, 8)):
+                         (pgvc.CHK_RACE | pgvc.CHK_OOB, 8), (pgvc.CHK_RACE | pgvc.CHK_OOB | fast, 32), (fast, 32)):
         ir.compile(bits=bits, checks=checks)
 
 
