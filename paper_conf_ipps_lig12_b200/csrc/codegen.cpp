@@ -585,15 +585,28 @@ struct Gen {
         }
         o << "      default: break;\n    }\n  }\n";
         // optimistic pass: reader check of a logged cell after the round's barrier
-        o << "  static __device__ __forceinline__ void fcheck_one(u32 step, PgT& t, u32 cell) {\n";
-        o << "    const u32 flat = cell & 0xFFFFFFu;\n    switch (cell >> 24) {\n";
-        for (size_t a = 0; a < K.arrays.size(); a++) {
-            const ArrayDecl& A = K.arrays[a];
-            if (!A.written || A.space == PRIVATE || !O.fast || !rda_[a]) continue;
-            o << "      case " << a << ": pg_fcheck_" << (A.space == SHARED ? "sh" : "gt") << "<" << a
-              << ">(step, t, flat); break;\n";
+        // (only arrays with tracked readers are logged: one such array needs no dispatch)
+        o << "  static __device__ __forceinline__ void fcheck_one(const PgC& C, PgT& t, u32 cell) {\n";
+        o << "    const u32 flat = cell & 0xFFFFFFu;\n";
+        {
+            std::vector<size_t> fa;
+            for (size_t a = 0; a < K.arrays.size(); a++) {
+                const ArrayDecl& A = K.arrays[a];
+                if (A.written && A.space != PRIVATE && O.fast && rda_[a]) fa.push_back(a);
+            }
+            auto call = [&](size_t a) {
+                return std::string("pg_fcheck_") + (K.arrays[a].space == SHARED ? "sh" : "gt") + "<" +
+                       std::to_string(a) + ">(C, t, flat);";
+            };
+            if (fa.size() == 1) {
+                o << "    " << call(fa[0]) << "\n";
+            } else {
+                o << "    switch (cell >> 24) {\n";
+                for (size_t a : fa) o << "      case " << a << ": " << call(a) << " break;\n";
+                o << "      default: break;\n    }\n";
+            }
         }
-        o << "      default: break;\n    }\n  }\n";
+        o << "  }\n";
         o << "  static __device__ __forceinline__ u32 seg(Frame& F, PgC& C, PgT& t, PgCold& c, u64* ss, u32 resume) {\n";
         o << "    switch (resume) {\n      case 0u: goto R0;\n";
         for (int k = 1; k <= seg_nsync; k++) o << "      case " << k << "u: goto R" << k << ";\n";

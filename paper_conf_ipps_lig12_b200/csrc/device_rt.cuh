@@ -115,7 +115,22 @@ struct PgC {        // CTA-uniform state
     u32 fuel;
     u32 ufuel;      // uniform-loop iterations this round
     u32 abort;      // PG_FAST: a race was flagged, the item stops (its instances are re-run exactly)
+    // derived from step / step0 once per round / block (pg_set_step, pg_set_step0)
+    u32 smin;       // (2^20-1 - step) << 12: owner / min-reader stamp of this round without the tid
+    u32 smax;       // step << 12: max-reader / max-writer stamp without the tid
+    u32 par;        // step & 1: reader-stamp set of the optimistic pass
+    u32 uthr;       // owner stamps >= uthr predate this block ("never written", X6)
 };
+__device__ __forceinline__ void pg_set_step(PgC& C, u32 s) {
+    C.step = s;
+    C.smin = (0xFFFFFu - s) << 12;
+    C.smax = s << 12;
+    C.par = s & 1u;
+}
+__device__ __forceinline__ void pg_set_step0(PgC& C, u32 s0) {
+    C.step0 = s0;
+    C.uthr = (0x100000u - s0) << 12;
+}
 
 struct PgT {        // hot per-emulated-thread state (kept in registers)
     u32 live;       // 0/1: not exited, and a real thread of a real instance and block
@@ -166,8 +181,8 @@ __device__ __noinline__ u32 pg_event(PgCold& c, u32 evm, u32 kind, u32 round, u3
 #define PG_EVENT(t, c, ...) ((t).evm |= pg_event((c), (t).evm, __VA_ARGS__))
 
 // stamps: step (20 bits, >= 1) and block-local tid (12 bits)
-__device__ __forceinline__ u32 pg_stamp_min(const PgC& C, const PgT& t) { return ((0xFFFFFu - C.step) << 12) | t.tlin; }
-__device__ __forceinline__ u32 pg_stamp_max(const PgC& C, const PgT& t) { return (C.step << 12) | t.tlin; }
+__device__ __forceinline__ u32 pg_stamp_min(const PgC& C, const PgT& t) { return C.smin | t.tlin; }
+__device__ __forceinline__ u32 pg_stamp_max(const PgC& C, const PgT& t) { return C.smax | t.tlin; }
 __device__ __forceinline__ u32 pg_owner_step(u32 own) { return 0xFFFFFu - (own >> 12); }
 
 __device__ __forceinline__ u32* pg_sh(const PgT& t, u32 off) { return (u32*)(pg_dsmem + t.sg + off); }
@@ -185,10 +200,6 @@ __device__ __forceinline__ u32* pg_sh(const PgT& t, u32 off) { return (u32*)(pg_
 // stamps of the cells it wrote - all reads of the round are visible then, whether they
 // came before or after the write - while the next round stamps the other set (RW).
 __shared__ u32 pg_sAbort;   // some thread of the CTA flagged (CTA-wide blocks)
-// reader stamps show a reader of round `step` other than this thread
-__device__ __forceinline__ u32 pg_fast_readers(u32 step, const PgT& t, u32 rmin, u32 rmax) {
-    return (rmax >> 12) == step && (((rmin & 0xFFFu) != t.tlin) | ((rmax & 0xFFFu) != t.tlin));
-}
 #endif
 
 // ------------------------------------------------------------------ bank / coalescing (X9, H6)
@@ -335,6 +346,42 @@ __device__ __forceinline__ u32 pg_poison_sh(const PgT& t, u32 rec, u32 flat) {
 // Shared array A: value and owner-stamp words in the group's region.
 // RD: reader stamps kept (race checks on, array read and written);
 // LOG: a load of A may follow a store to A in the same round (own-write lookup).
+#if PG_FAST
+// cold path of a shared load: out of bounds or never written (X5/X6): poison value and
+// the event (returned as value | event bits << 32)
+__device__ __noinline__ u64 pg_ld_sh_cold(PgCold& c, u32 evm, u64 seed, u32 blk, u32 rec, u32 flat, u32 round,
+                                         u32 gtid, u32 site, u32 oob) {
+    const u32 pv = pg_m(pg_rand32(seed, 0x8000u + (rec - 0x100u), ((u64)blk << 20) + flat));
+    u32 bits = 0u;
+#if PG_OOBCHK
+    bits = pg_event(c, evm, oob ? PGK_OOB : PGK_UNINIT, round, rec, flat, gtid, PG_NEVER, site, pv, 0);
+#endif
+    return (u64)pv | ((u64)bits << 32);
+}
+template <int A, bool RD, bool LOG>
+__device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site) {
+    const u32 inb = flat < PG_SH(A, size);
+#if PG_BANKCHK
+    t.evm |= pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, t.evm, ss, pe & inb, PG_ARR(A).rec_id, flat, site);
+#endif
+    u32 own = 0u, v = 0u;
+    if (pe & inb) {
+        if (RD && PG_T > 1u) {
+            const u32 so = C.par * PG_SH(A, size) + flat;
+            atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + so, C.smin | t.tlin);
+            atomicMax(pg_sh(t, PG_SH(A, s_rmax)) + so, C.smax | t.tlin);
+        }
+        own = pg_sh(t, PG_SH(A, s_own))[flat];
+        v = pg_sh(t, PG_SH(A, s_val))[flat];
+    }
+    if (pe & ((inb ^ 1u) | (u32)(own >= C.uthr))) {
+        const u64 r = pg_ld_sh_cold(c, t.evm, t.seed, t.blk, PG_ARR(A).rec_id, flat, C.round, t.gtid, site, inb ^ 1u);
+        t.evm |= (u32)(r >> 32);
+        v = (u32)r;
+    }
+    return v;
+}
+#else
 template <int A, bool RD, bool LOG>
 __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site) {
     const u32 inb = flat < PG_SH(A, size);
@@ -349,14 +396,6 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
 #endif
         return pv;
     }
-#if PG_FAST
-    if (RD && PG_T > 1u) {
-        const u32 so = (C.step & 1u) * PG_SH(A, size) + flat;
-        atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + so, pg_stamp_min(C, t));
-        atomicMax(pg_sh(t, PG_SH(A, s_rmax)) + so, pg_stamp_max(C, t));
-    }
-    const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
-#else
 #if PG_RACECHK
     if (RD && PG_T > 1u) {
         atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + flat, pg_stamp_min(C, t));
@@ -371,8 +410,7 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
         return v;
     }
     const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
-#endif
-    if (pg_owner_step(own) < C.step0) {  // never written in this block (X6)
+    if (own >= C.uthr) {  // never written in this block (X6)
         const u32 pv = pg_poison_sh(t, PG_ARR(A).rec_id, flat);
 #if PG_OOBCHK
         PG_EVENT(t, c, PGK_UNINIT, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
@@ -388,6 +426,7 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
 #endif
     return pg_sh(t, PG_SH(A, s_val))[flat];
 }
+#endif
 
 #if PG_FAST
 // write log of the optimistic pass: cells whose readers are checked after the barrier
@@ -411,10 +450,10 @@ __device__ __forceinline__ void pg_fcount(PgT& t) {
 template <int A, bool RDA>
 __device__ __forceinline__ void pg_commit_sh(const PgC& C, PgT& t, PgCold& c, u32 flat, u32 val) {
     u32* own = pg_sh(t, PG_SH(A, s_own)) + flat;
-    const u32 me = pg_stamp_min(C, t);
+    const u32 me = C.smin | t.tlin;
     if (PG_T > 1u) {
         const u32 old = atomicMin(own, me);
-        t.fl |= (old != me) & ((old >> 12) == (me >> 12));   // a second writer this round (WW)
+        t.fl |= (old ^ me) - 1u < 0xFFFu;   // another writer's stamp of this round (WW)
         if (RDA) pg_flog(t, c, ((u32)A << 24) | flat);
     } else {
         *own = me;
@@ -423,22 +462,29 @@ __device__ __forceinline__ void pg_commit_sh(const PgC& C, PgT& t, PgCold& c, u3
     pg_fcount(t);
 }
 // after the round's barrier: readers of a cell this thread wrote in round `step`
-template <int A>
-__device__ __forceinline__ void pg_fcheck_sh(u32 step, PgT& t, u32 flat) {
-    const u32 so = (step & 1u) * PG_SH(A, size) + flat;
-    t.fl |= pg_fast_readers(step, t, pg_sh(t, PG_SH(A, s_rmin))[so], pg_sh(t, PG_SH(A, s_rmax))[so]);
+// readers of the round other than this thread: the max reader stamp is of this round and
+// the min / max reader stamps are not both this thread's
+__device__ __forceinline__ u32 pg_fast_rw(const PgC& C, const PgT& t, u32 rmin, u32 rmax) {
+    const u32 a = rmax ^ (C.smax | t.tlin);
+    return (a < 0x1000u) & ((a | (rmin ^ (C.smin | t.tlin))) != 0u);
 }
 template <int A>
-__device__ __forceinline__ void pg_fcheck_gt(u32 step, PgT& t, u32 flat) {
-    const u64 so = (u64)(step & 1u) * PG_ARR(A).size + flat;
-    t.fl |= pg_fast_readers(step, t, t.arena[PG_ARR(A).off_rmin + so], t.arena[PG_ARR(A).off_rmax + so]);
+__device__ __forceinline__ void pg_fcheck_sh(const PgC& C, PgT& t, u32 flat) {
+    const u32 so = C.par * PG_SH(A, size) + flat;
+    t.fl |= pg_fast_rw(C, t, pg_sh(t, PG_SH(A, s_rmin))[so], pg_sh(t, PG_SH(A, s_rmax))[so]);
 }
+template <int A>
+__device__ __forceinline__ void pg_fcheck_gt(const PgC& C, PgT& t, u32 flat) {
+    const u64 so = (u64)C.par * PG_ARR(A).size + flat;
+    t.fl |= pg_fast_rw(C, t, t.arena[PG_ARR(A).off_rmin + so], t.arena[PG_ARR(A).off_rmax + so]);
+}
+// (C still describes the round just finished)
 template <class K>
-__device__ __forceinline__ void pg_fcheck_all(u32 step, PgT& t, PgCold& c) {
+__device__ __forceinline__ void pg_fcheck_all(const PgC& C, PgT& t, PgCold& c) {
     const u32 n = t.nlog & 0xFFFFu;
     if (n == 0u) return;
-    K::fcheck_one(step, t, t.l0cell);
-    for (u32 i = 1; i < n; i++) K::fcheck_one(step, t, c.lcell[i]);
+    K::fcheck_one(C, t, t.l0cell);
+    for (u32 i = 1; i < n; i++) K::fcheck_one(C, t, c.lcell[i]);
 }
 #endif
 
@@ -491,9 +537,9 @@ __device__ __forceinline__ u32 pg_ld_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
     pg_xb_mark<A>(t, flat);
 #if PG_FAST
     if (RD && PG_T > 1u) {
-        const u64 so = (u64)(C.step & 1u) * PG_ARR(A).size + flat;
-        atomicMin(t.arena + PG_ARR(A).off_rmin + so, pg_stamp_min(C, t));
-        atomicMax(t.arena + PG_ARR(A).off_rmax + so, pg_stamp_max(C, t));
+        const u64 so = (u64)C.par * PG_ARR(A).size + flat;
+        atomicMin(t.arena + PG_ARR(A).off_rmin + so, C.smin | t.tlin);
+        atomicMax(t.arena + PG_ARR(A).off_rmax + so, C.smax | t.tlin);
     }
     return t.arena[PG_ARR(A).off_val + flat];
 #else
@@ -535,10 +581,10 @@ __device__ __forceinline__ void pg_st_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32
 #if PG_FAST
     {
         u32* own = t.arena + PG_ARR(A).off_own + flat;
-        const u32 me = pg_stamp_min(C, t);
+        const u32 me = C.smin | t.tlin;
         if (PG_T > 1u) {
             const u32 old = atomicMin(own, me);
-            t.fl |= (old != me) & ((old >> 12) == (me >> 12));
+            t.fl |= (old ^ me) - 1u < 0xFFFu;
             if (RDA) pg_flog(t, c, ((u32)A << 24) | flat);
         } else {
             *own = me;
@@ -730,7 +776,7 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
     if (warp_blocks) __syncwarp();
     if (LAST) {
         if (!warp_blocks) __syncthreads();
-        pg_fcheck_all<K>(C.step, t, c);
+        pg_fcheck_all<K>(C, t, c);
         return false;
     }
     int more;
@@ -746,9 +792,9 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
         t.fl = 1u;
         return false;
     }
-    pg_fcheck_all<K>(C.step, t, c);   // (flags found here stop the item at the next round end)
+    pg_fcheck_all<K>(C, t, c);   // (flags found here stop the item at the next round end)
     if (!more) return false;
-    C.step++;
+    pg_set_step(C, C.step + 1u);
     C.ufuel = 0;
     t.nlog = 0;
     t.fuel = 0;
@@ -767,7 +813,7 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
     if (LAST) return false;
     const int more = warp_blocks ? __any_sync(PG_FULL, t.live) : __syncthreads_or((int)t.live);
     if (!more) return false;
-    C.step++;
+    pg_set_step(C, C.step + 1u);
     C.ufuel = 0;
     t.nlog = 0;
     t.fuel = 0;
@@ -982,7 +1028,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     for (u32 i = threadIdx.x; i < PG_PK; i += blockDim.x) s_grounds[i] = 0;
 
     PgC C;
-    C.step = 0;
+    pg_set_step(C, 0u);
     C.abort = 0;
 #if PG_FAST
     if (threadIdx.x == 0) pg_sAbort = 0u;   // (published by the barrier below)
@@ -1039,7 +1085,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     for (u32 st = 0; st < nsteps; st++) {
         const u32 blk = pg_sW.blk0 + st * GB + bs;
         const u32 blk_ok = blk < pg_sW.blk1;
-        C.step0 = C.step + 1u;
+        pg_set_step0(C, C.step + 1u);
         u32 alive_rounds = 0;  // rounds this thread entered alive (X19: group rounds = max over threads)
 #pragma unroll
         for (u32 v = 0; v < PG_VMAX; v++) {
@@ -1069,7 +1115,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 #if PG_VMAX == 1
         {   // rounds inline: K::run ends each round at its barrier (pg_round_end)
             PgT& t = T[0];
-            C.step++;
+            pg_set_step(C, C.step + 1u);
             C.ufuel = 0;
             t.nlog = 0;
             t.fuel = 0;
@@ -1079,7 +1125,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 #else
         u32 resume = 0;
         for (;;) {
-            C.step++;
+            pg_set_step(C, C.step + 1u);
             C.ufuel = 0;
             u32 r = PG_END;
             u32 any_start = 0;
@@ -1140,7 +1186,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
-                pg_fcheck_all<K>(C.step, T[v], Cd[v]);
+                pg_fcheck_all<K>(C, T[v], Cd[v]);
             }
 #else
             const int more = warp_blocks ? __any_sync(PG_FULL, any) : __syncthreads_or((int)any);
