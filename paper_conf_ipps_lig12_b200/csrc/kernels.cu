@@ -23,20 +23,48 @@ __device__ __forceinline__ u32 init_value(u32 mode, u32 range, u32 mask, u64 see
 // stride over the words.
 // With `flags`, only the jobs of region `only_target` and only flagged instances are
 // (re-)initialised: the exact re-run of the instances the optimistic pass flagged.
+// Work units of the per-(job, instance) kernels K1/K2b/K3: a CTA per instance for arrays
+// of more than kSmallN words, else a warp per instance (most C1-C4 output arrays hold a
+// few words: a CTA of idle threads per instance would cost more than the words).
+constexpr u32 kSmallN = 512u;
+// Large arrays are cut into chunks of kChunk words, one CTA per (instance, chunk), so one
+// instance's words are spread over many SMs.
+constexpr u32 kChunk = 65536u;
+struct Units {
+    u32 first, step, tid, nthr;   // unit loop (first, step) and word loop (tid, nthr)
+    u32 nchunk;                   // units per instance
+};
+__device__ __forceinline__ Units pg_units(u32 n) {
+    if (n > kSmallN) return Units{blockIdx.x, gridDim.x, threadIdx.x, blockDim.x, (n + kChunk - 1u) / kChunk};
+    const u32 nw = blockDim.x >> 5;
+    return Units{blockIdx.x * nw + (threadIdx.x >> 5), gridDim.x * nw, threadIdx.x & 31u, 32u, 1u};
+}
+// words [w0, w1) of unit `un` (instance un / nchunk)
+__device__ __forceinline__ void pg_unit_words(const Units& u, u32 un, u32 n, u32& inst, u32& w0, u32& w1) {
+    inst = un / u.nchunk;
+    w0 = (un - inst * u.nchunk) * kChunk;
+    w1 = u.nchunk == 1u ? n : min(n, w0 + kChunk);
+    if (u.nchunk == 1u) w0 = 0u;
+}
+
+// (with `flags`, only flagged instances are (re-)initialised: the exact re-run of the
+// instances the optimistic pass flagged)
 __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ jobs, u32* arena_s, u32* arena_t,
                                                      u32* input, u64 seed_base, u32 mode, u32 range, u32 mask,
-                                                     const u32* flags, u32 only_target) {
+                                                     const u32* flags) {
     const PgFill f = jobs[blockIdx.y];
-    if (flags && f.target != only_target) return;
     u32* region = f.target == 0 ? arena_s : f.target == 1 ? arena_t : input;
-    for (u32 inst = blockIdx.x; inst < f.n_inst; inst += gridDim.x) {
+    const Units u = pg_units(f.n);
+    for (u32 un = u.first; un < f.n_inst * u.nchunk; un += u.step) {
+        u32 inst, w0, w1;
+        pg_unit_words(u, un, f.n, inst, w0, w1);
         if (flags && !flags[f.inst0 + inst]) continue;
         u32* base = region + f.dst + (u64)inst * f.stride;
         const u64 seed = seed_base + (u64)f.j0 + (u64)inst * f.jstep;
         if (f.op == PGF_CONST) {
-            for (u32 i = threadIdx.x; i < f.n; i += blockDim.x) base[i] = f.value;
+            for (u32 i = w0 + u.tid; i < w1; i += u.nthr) base[i] = f.value;
         } else {  // PGF_INPUT (initial values of an input region or of a written array)
-            for (u32 i = threadIdx.x; i < f.n; i += blockDim.x) base[i] = init_value(mode, range, mask, seed, f.gid, i);
+            for (u32 i = w0 + u.tid; i < w1; i += u.nthr) base[i] = init_value(mode, range, mask, seed, f.gid, i);
         }
     }
 }
@@ -53,12 +81,32 @@ __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs
     const PgCmp c = jobs[blockIdx.y];
     const u32* rs = c.src_kind == 0 ? arena_s : input;
     const u32* rt = c.tgt_kind == 0 ? arena_t : input;
-    for (u32 inst = blockIdx.x; inst < c.n_inst; inst += gridDim.x) {
+    if (c.n <= kSmallN) {   // a warp per instance
+        const Units u = pg_units(c.n);
+        for (u32 inst = u.first; inst < c.n_inst; inst += u.step) {
+            const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
+            u32 cnt = 0, mn = PG_NEVER;
+            for (u32 i = u.tid; i < c.n; i += 32u) {
+                if (cmp_val(rs, c.src_kind, so, i) != cmp_val(rt, c.tgt_kind, to, i)) { cnt++; mn = min(mn, i); }
+            }
+            cnt = __reduce_add_sync(0xffffffffu, cnt);
+            mn = __reduce_min_sync(0xffffffffu, mn);
+            if (u.tid == 0 && cnt) {
+                atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step].count, (u64)cnt);
+                atomicMin(&mm_key[c.inst0 + inst], ((u64)c.gid << 32) | mn);
+            }
+        }
+        return;
+    }
+    const Units u = pg_units(c.n);
+    for (u32 un = u.first; un < c.n_inst * u.nchunk; un += u.step) {
+        u32 inst, w0, w1;
+        pg_unit_words(u, un, c.n, inst, w0, w1);
         if (threadIdx.x == 0) { s_cnt = 0; s_min = PG_NEVER; }
         __syncthreads();
         const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
         u32 cnt = 0, mn = PG_NEVER;
-        for (u32 i = threadIdx.x; i < c.n; i += blockDim.x) {
+        for (u32 i = w0 + threadIdx.x; i < w1; i += blockDim.x) {
             if (cmp_val(rs, c.src_kind, so, i) != cmp_val(rt, c.tgt_kind, to, i)) { cnt++; mn = min(mn, i); }
         }
         cnt = __reduce_add_sync(0xffffffffu, cnt);
@@ -102,12 +150,28 @@ __global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__
 // accessed by two blocks (X4 XB) - the block-parallel pass is not exact there.
 __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ jobs, const u32* arena, u32* flags) {
     const PgXb j = jobs[blockIdx.y];
-    for (u32 inst = blockIdx.x; inst < j.n_inst; inst += gridDim.x) {
+    if (j.n <= kSmallN) {   // a warp per instance
+        const Units u = pg_units(j.n);
+        for (u32 inst = u.first; inst < j.n_inst; inst += u.step) {
+            const u64 base = (u64)inst * j.stride;
+            u32 hit = 0;
+            for (u32 i = u.tid; i < j.n; i += 32u) {
+                const u32 xf = arena[j.xf + base + i], xl = arena[j.xl + base + i];
+                hit |= (xl != 0u && xf != xl && arena[j.lw + base + i] != 0u);
+            }
+            if (__any_sync(0xffffffffu, hit) && u.tid == 0) flags[j.inst0 + inst] = 1u;
+        }
+        return;
+    }
+    const Units u = pg_units(j.n);
+    for (u32 un = u.first; un < j.n_inst * u.nchunk; un += u.step) {
+        u32 inst, w0, w1;
+        pg_unit_words(u, un, j.n, inst, w0, w1);
         const u64 base = (u64)inst * j.stride;
         u32 hit = 0;
-        for (u32 i = threadIdx.x; i < j.n; i += blockDim.x) {
-            const u32 xf = arena[j.xf + base + i], xl = arena[j.xl + base + i];
-            hit |= (xl != 0u && xf != xl && arena[j.lw + base + i] != 0u);
+        for (u32 i = w0 + threadIdx.x; i < w1; i += blockDim.x) {
+            const u32 xf = arena[j.xf + base + i], xl = arena[j.xl + base + i], lw = arena[j.lw + base + i];
+            hit |= (xl != 0u) & (xf != xl) & (lw != 0u);
         }
         if (__syncthreads_or((int)hit) && threadIdx.x == 0) flags[j.inst0 + inst] = 1u;
     }
@@ -350,14 +414,16 @@ __global__ void __launch_bounds__(1024) pg_count_reduce(const u64* inst_cnt, u32
 // ------------------------------------------------------------------ host wrappers (C++ linkage, used by api.cpp)
 namespace pgk {
 
+// grid.x of the per-(job, instance) kernels: enough CTAs for a CTA per instance, capped
+// (re-initialisation of flagged instances: a few CTAs per job walk its instances)
+static u32 units_grid(u32 max_inst, u32 cap) { return max_inst < cap ? (max_inst ? max_inst : 1u) : cap; }
+
 cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 max_inst, u32* arena_s, u32* arena_t, u32* input,
-                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags,
-                       u32 only_target) {
+                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags) {
     for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
         const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
-        dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
-        pg_gen_inputs<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, seed_base, mode, range, mask, flags,
-                                            only_target);
+        dim3 grid(units_grid(max_inst, flags ? 8u : 1024u), nj);
+        pg_gen_inputs<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, seed_base, mode, range, mask, flags);
     }
     return cudaGetLastError();
 }
