@@ -28,6 +28,89 @@ std::string hex(uint32_t v) {
     return b;
 }
 
+// ---------------------------------------------------------------- seed-oblivious analysis
+// Input dependence ("taint"): a load's value depends on the seed; so does every expression
+// over it and every variable assigned one (fixed point).  The kernel is seed-oblivious when
+// no address, store guard, branch or loop condition is tainted: then all seeds of a launch
+// take the same accesses in the same rounds (the stamps, races and instance counts agree)
+// and one lane can carry several seeds' values (multi-seed lanes).
+struct Taint {
+    std::vector<bool> tv;
+    bool ok = true;
+    bool tainted(const Node* n) const {
+        if (!n) return false;
+        if (n->kind == NK::Elem) return true;
+        if (n->kind == NK::Var) return tv[(size_t)n->ref];
+        for (const Node* k : n->kids)
+            if (tainted(k)) return true;
+        return false;
+    }
+    static bool has_load(const Node* n) {
+        if (!n) return false;
+        if (n->kind == NK::Elem) return true;
+        for (const Node* k : n->kids)
+            if (has_load(k)) return true;
+        return false;
+    }
+    bool prop(const Stmt* s) {
+        if (!s) return false;
+        bool ch = false;
+        switch (s->kind) {
+        case SK::Seq:
+            for (const Stmt* c : s->seq) ch |= prop(c);
+            break;
+        case SK::Assign:
+            if (!tv[(size_t)s->var] && tainted(s->value)) tv[(size_t)s->var] = ch = true;
+            break;
+        case SK::If: ch |= prop(s->body); ch |= prop(s->other); break;
+        case SK::Loop: ch |= prop(s->init); ch |= prop(s->body); ch |= prop(s->step); break;
+        default: break;
+        }
+        return ch;
+    }
+    void check_expr(const Node* n) {
+        if (!n) return;
+        if (n->kind == NK::Elem)
+            for (const Node* i : n->kids)
+                if (tainted(i)) ok = false;   // input-dependent address
+        if ((n->kind == NK::LAnd || n->kind == NK::LOr || n->kind == NK::Select) && tainted(n->kids[0]))
+            for (size_t i = 1; i < n->kids.size(); i++)
+                if (has_load(n->kids[i])) ok = false;   // input-dependent load guard
+        for (const Node* k : n->kids) check_expr(k);
+    }
+    void check(const Stmt* s) {
+        if (!s) return;
+        switch (s->kind) {
+        case SK::Seq:
+            for (const Stmt* c : s->seq) check(c);
+            break;
+        case SK::Assign: check_expr(s->value); break;
+        case SK::Store:
+            for (const Node* i : s->index) {
+                if (tainted(i)) ok = false;
+                check_expr(i);
+            }
+            check_expr(s->value);
+            break;
+        case SK::PrivDecl: ok = false; break;
+        case SK::If:
+            if (tainted(s->cond)) ok = false;   // input-dependent guard of the branches' accesses
+            check_expr(s->cond);
+            check(s->body);
+            check(s->other);
+            break;
+        case SK::Loop:
+            check(s->init);
+            if (tainted(s->cond)) ok = false;
+            check_expr(s->cond);
+            check(s->body);
+            check(s->step);
+            break;
+        default: break;
+        }
+    }
+};
+
 struct Gen {
     const Kernel& K;
     const CodegenOptions& O;
@@ -183,6 +266,26 @@ struct Gen {
     }
 
     std::string tmp(const char* p = "t") { return std::string("_") + p + std::to_string(ntmp++); }
+
+    // ---------------------------------------------------------------- multi-seed lanes
+    // (O.ms > 1) tainted values are arrays of PG_MS words, one per seed; untainted ones
+    // (addresses, guards, loop counters) stay scalar and are computed once for all seeds
+    std::vector<bool> tvar_;
+    std::set<std::string> tnames_;   // temporaries / frame slots holding PG_MS copies
+    bool ms() const { return O.ms > 1; }
+    bool tn(const std::string& x) const { return ms() && tnames_.count(x) != 0; }
+    std::string at(const std::string& x) const { return tn(x) ? x + "[_s]" : x; }
+    std::string defv(const std::string& e) {   // e refers to its operands through at()
+        std::string r = tmp();
+        line("u32 " + r + "[PG_MS]; PG_S_LOOP " + r + "[_s] = " + e + ";");
+        tnames_.insert(r);
+        return r;
+    }
+    std::string def2(bool t, const std::string& e) { return t ? defv(e) : def(e); }
+    std::string vec(const std::string& x) {   // a PG_MS-word copy of x (store operands)
+        if (tn(x)) return x;
+        return defv(x);
+    }
     int label() { return nlabel++; }
     void line(const std::string& s) { body << "  " << s << "\n"; }
     bool uniform_ctx() const { return preds.empty(); }
@@ -239,13 +342,23 @@ struct Gen {
             std::string f = flat_index(n, n->ref, pr);
             std::string r = tmp();
             std::string A = std::to_string(n->ref), S = std::to_string(n->site) + "u";
+            const std::string st = stamps_needed(n) ? "true" : "false", lg = log_[(size_t)n->ref] ? "true" : "false";
+            if (ms()) {   // (seed-oblivious: shared or global, never private)
+                line("u32 " + r + "[PG_MS];");
+                tnames_.insert(r);
+                if (a.space == SHARED)
+                    line("pg_ld_sh_ms<" + A + ", " + st + ", " + lg + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ", " + r + ");");
+                else if (a.written)
+                    line("pg_ld_gt_ms<" + A + ", " + st + ", " + lg + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ", " + r + ");");
+                else
+                    line("pg_ld_gi_ms<" + A + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ", " + r + ");");
+                return r;
+            }
             if (a.space == SHARED) {
-                line("u32 " + r + " = pg_ld_sh<" + A + ", " + (stamps_needed(n) ? "true" : "false") + ", " +
-                     (log_[(size_t)n->ref] ? "true" : "false") + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
+                line("u32 " + r + " = pg_ld_sh<" + A + ", " + st + ", " + lg + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
             } else if (a.space == GLOBAL) {
                 if (a.written)
-                    line("u32 " + r + " = pg_ld_gt<" + A + ", " + (stamps_needed(n) ? "true" : "false") + ", " +
-                         (log_[(size_t)n->ref] ? "true" : "false") + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
+                    line("u32 " + r + " = pg_ld_gt<" + A + ", " + st + ", " + lg + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
                 else
                     line("u32 " + r + " = pg_ld_gi<" + A + ">(C, t, c, ss, " + pr + ", " + f + ", " + S + ");");
             } else {
@@ -255,56 +368,66 @@ struct Gen {
             }
             return r;
         }
-        case NK::Neg: return def("pg_neg(" + ex(n->kids[0], pr) + ")");
-        case NK::BitNot: return def("pg_not(" + ex(n->kids[0], pr) + ")");
-        case NK::LogNot: return def("(u32)(" + ex(n->kids[0], pr) + " == 0u)");
+        case NK::Neg: { std::string a = ex(n->kids[0], pr); return def2(tn(a), "pg_neg(" + at(a) + ")"); }
+        case NK::BitNot: { std::string a = ex(n->kids[0], pr); return def2(tn(a), "pg_not(" + at(a) + ")"); }
+        case NK::LogNot: { std::string a = ex(n->kids[0], pr); return def2(tn(a), "(u32)(" + at(a) + " == 0u)"); }
         case NK::Cast: return ex(n->kids[0], pr);
-        case NK::LAnd: {
-            std::string a = def("(u32)(" + ex(n->kids[0], pr) + " != 0u)");
-            std::string p = def("(" + pr + ") & " + a);
-            std::string b = ex(n->kids[1], p);
-            return def(a + " & (u32)(" + b + " != 0u)");
-        }
+        case NK::LAnd:
         case NK::LOr: {
-            std::string a = def("(u32)(" + ex(n->kids[0], pr) + " != 0u)");
-            std::string p = def("(" + pr + ") & (" + a + " ^ 1u)");
+            const bool land = n->kind == NK::LAnd;
+            std::string x = ex(n->kids[0], pr);
+            std::string a = def2(tn(x), "(u32)(" + at(x) + " != 0u)");
+            if (tn(a)) {   // input-dependent condition: the other operand has no loads (seed_oblivious)
+                std::string b = ex(n->kids[1], pr);
+                return defv(at(a) + (land ? " & " : " | ") + "(u32)(" + at(b) + " != 0u)");
+            }
+            std::string p = def(land ? "(" + pr + ") & " + a : "(" + pr + ") & (" + a + " ^ 1u)");
             std::string b = ex(n->kids[1], p);
-            return def(a + " | (u32)(" + b + " != 0u)");
+            return def2(tn(b), a + (land ? " & " : " | ") + "(u32)(" + at(b) + " != 0u)");
         }
         case NK::Select: {
-            std::string c = def("(u32)(" + ex(n->kids[0], pr) + " != 0u)");
+            std::string cx = ex(n->kids[0], pr);
+            std::string c = def2(tn(cx), "(u32)(" + at(cx) + " != 0u)");
+            if (tn(c)) {
+                std::string x = ex(n->kids[1], pr), y = ex(n->kids[2], pr);
+                return defv(at(c) + " ? " + at(x) + " : " + at(y));
+            }
             std::string p1 = def("(" + pr + ") & " + c);
             std::string p0 = def("(" + pr + ") & (" + c + " ^ 1u)");
             std::string x = ex(n->kids[1], p1);
             std::string y = ex(n->kids[2], p0);
-            return def(c + " ? " + x + " : " + y);
+            return def2(tn(x) || tn(y), c + " ? " + at(x) + " : " + at(y));
         }
         case NK::Min:
         case NK::Max: {
-            std::string a = ex(n->kids[0], pr), b = ex(n->kids[1], pr);
+            std::string a0 = ex(n->kids[0], pr), b0 = ex(n->kids[1], pr);
+            const bool T = tn(a0) || tn(b0);
+            std::string a = at(a0), b = at(b0);
             std::string lt = n->opty == Ty::U32 ? "(" + a + " < " + b + ")" : "pg_slt(" + a + ", " + b + ")";
-            return def(n->kind == NK::Min ? lt + " ? " + a + " : " + b : lt + " ? " + b + " : " + a);
+            return def2(T, n->kind == NK::Min ? lt + " ? " + a + " : " + b : lt + " ? " + b + " : " + a);
         }
         case NK::Bin: {
-            std::string a = ex(n->kids[0], pr), b = ex(n->kids[1], pr);
+            std::string a0 = ex(n->kids[0], pr), b0 = ex(n->kids[1], pr);
+            const bool T = tn(a0) || tn(b0);
+            std::string a = at(a0), b = at(b0);
             bool u = n->opty == Ty::U32;
             switch (n->op) {
-            case Bop::Add: return def("pg_add(" + a + ", " + b + ")");
-            case Bop::Sub: return def("pg_sub(" + a + ", " + b + ")");
-            case Bop::Mul: return def("pg_mul(" + a + ", " + b + ")");
-            case Bop::Div: return def(std::string(u ? "pg_udiv(" : "pg_sdiv(") + a + ", " + b + ")");
-            case Bop::Rem: return def(std::string(u ? "pg_urem(" : "pg_srem(") + a + ", " + b + ")");
-            case Bop::Shl: return def("pg_shl(" + a + ", " + b + ")");
-            case Bop::Shr: return def(std::string(u ? "pg_lshr(" : "pg_ashr(") + a + ", " + b + ")");
-            case Bop::And: return def("(" + a + " & " + b + ")");
-            case Bop::Or: return def("(" + a + " | " + b + ")");
-            case Bop::Xor: return def("(" + a + " ^ " + b + ")");
-            case Bop::Lt: return def(u ? "(u32)(" + a + " < " + b + ")" : "pg_slt(" + a + ", " + b + ")");
-            case Bop::Le: return def(u ? "(u32)(" + a + " <= " + b + ")" : "pg_sle(" + a + ", " + b + ")");
-            case Bop::Gt: return def(u ? "(u32)(" + a + " > " + b + ")" : "pg_slt(" + b + ", " + a + ")");
-            case Bop::Ge: return def(u ? "(u32)(" + a + " >= " + b + ")" : "pg_sle(" + b + ", " + a + ")");
-            case Bop::Eq: return def("(u32)(" + a + " == " + b + ")");
-            case Bop::Ne: return def("(u32)(" + a + " != " + b + ")");
+            case Bop::Add: return def2(T, "pg_add(" + a + ", " + b + ")");
+            case Bop::Sub: return def2(T, "pg_sub(" + a + ", " + b + ")");
+            case Bop::Mul: return def2(T, "pg_mul(" + a + ", " + b + ")");
+            case Bop::Div: return def2(T, std::string(u ? "pg_udiv(" : "pg_sdiv(") + a + ", " + b + ")");
+            case Bop::Rem: return def2(T, std::string(u ? "pg_urem(" : "pg_srem(") + a + ", " + b + ")");
+            case Bop::Shl: return def2(T, "pg_shl(" + a + ", " + b + ")");
+            case Bop::Shr: return def2(T, std::string(u ? "pg_lshr(" : "pg_ashr(") + a + ", " + b + ")");
+            case Bop::And: return def2(T, "(" + a + " & " + b + ")");
+            case Bop::Or: return def2(T, "(" + a + " | " + b + ")");
+            case Bop::Xor: return def2(T, "(" + a + " ^ " + b + ")");
+            case Bop::Lt: return def2(T, u ? "(u32)(" + a + " < " + b + ")" : "pg_slt(" + a + ", " + b + ")");
+            case Bop::Le: return def2(T, u ? "(u32)(" + a + " <= " + b + ")" : "pg_sle(" + a + ", " + b + ")");
+            case Bop::Gt: return def2(T, u ? "(u32)(" + a + " > " + b + ")" : "pg_slt(" + b + ", " + a + ")");
+            case Bop::Ge: return def2(T, u ? "(u32)(" + a + " >= " + b + ")" : "pg_sle(" + b + ", " + a + ")");
+            case Bop::Eq: return def2(T, "(u32)(" + a + " == " + b + ")");
+            case Bop::Ne: return def2(T, "(u32)(" + a + " != " + b + ")");
             }
         }
         }
@@ -330,8 +453,14 @@ struct Gen {
             line("{");
             std::string v = ex(s->value, eff());
             std::string dst = "F.v" + std::to_string(s->var);
-            if (uniform_ctx()) line(dst + " = " + v + ";");
-            else line(dst + " = " + eff() + " ? " + v + " : " + dst + ";");
+            if (tn(dst)) {
+                if (uniform_ctx()) line("PG_S_LOOP " + dst + "[_s] = " + at(v) + ";");
+                else line("PG_S_LOOP " + dst + "[_s] = " + eff() + " ? " + at(v) + " : " + dst + "[_s];");
+            } else if (uniform_ctx()) {
+                line(dst + " = " + v + ";");
+            } else {
+                line(dst + " = " + eff() + " ? " + v + " : " + dst + ";");
+            }
             line("}");
             return;
         }
@@ -344,6 +473,13 @@ struct Gen {
             std::string f = flat_index(&tmpn, s->arr, pe);
             std::string v = ex(s->value, pe);
             std::string A = std::to_string(s->arr), S = std::to_string(s->site) + "u";
+            if (ms()) {
+                v = vec(v);
+                line(std::string(a.space == SHARED ? "pg_st_sh_ms<" : "pg_st_gt_ms<") + A + ", " + rda(s->arr) +
+                     ">(C, t, c, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
+                line("}");
+                return;
+            }
             if (a.space == SHARED)
                 line("pg_st_sh<" + A + ", " + rda(s->arr) + ">(C, t, c, ss, " + pe + ", " + f + ", " + v + ", " + S + ");");
             else if (a.space == GLOBAL)
@@ -511,6 +647,12 @@ struct Gen {
             lw_stmt(K.body, st);
         }
         seg_run();
+        tvar_.assign(K.vars.size(), false);
+        if (ms()) {
+            if (!seed_oblivious(K, &tvar_)) throw FrontError(-7, "multi-seed variant of a kernel that is not seed-oblivious");
+            for (size_t i = 0; i < K.vars.size(); i++)
+                if (tvar_[i]) tnames_.insert("F.v" + std::to_string(i));
+        }
         rda_.assign(K.arrays.size(), false);
         for (const auto& ld : seg_ld_)
             if (stamps_needed(ld.first)) rda_[(size_t)ld.first->ref] = true;
@@ -546,13 +688,15 @@ struct Gen {
         o << "#define PG_LOCKSTEP " << ((O.checks & 64) ? 1 : 0) << "\n";
         o << "#define PG_FAST " << (O.fast ? 1 : 0) << "\n";
         o << "#define PG_WMAX " << O.wmax << "\n";
+        o << "#define PG_MS " << (ms() ? O.ms : 1u) << "\n";
         o << "#define PG_NSTATS " << std::max<size_t>(1, K.sites.size()) << "\n";
         o << "#ifndef PG_VMAX\n#define PG_VMAX 1\n#endif\n";
         o << "#include \"pg_device_rt.cuh\"\n\n";
         o << "// kernel " << K.name << "\n";
         o << "struct PgK {\n  struct Frame {\n";
         for (size_t i = 0; i < K.vars.size(); i++)
-            o << "    u32 v" << i << ";  // " << K.vars[i].name << (K.vars[i].uniform ? " (uniform)" : "") << "\n";
+            o << "    u32 v" << i << (tvar_[i] ? "[PG_MS]" : "") << ";  // " << K.vars[i].name
+              << (K.vars[i].uniform ? " (uniform)" : "") << (tvar_[i] && ms() ? " (per seed)" : "") << "\n";
         for (const ArrayDecl& a : K.arrays)
             if (a.space == PRIVATE) o << "    u32 p" << a.slot << "[" << priv_size(a) << "];  // " << a.name << "\n";
         o << "    u32 pad_;\n  };\n";
@@ -560,6 +704,8 @@ struct Gen {
         for (size_t i = 0; i < K.vars.size(); i++) {
             if (K.vars[i].scalar)
                 o << "    F.v" << i << " = pg_m((u32)pg_sL.scal[" << K.vars[i].scalar_index << "]);\n";
+            else if (ms() && tvar_[i])
+                o << "    PG_S_LOOP F.v" << i << "[_s] = 0u;\n";
             else
                 o << "    F.v" << i << " = 0u;\n";
         }
@@ -624,6 +770,18 @@ struct Gen {
 };
 
 }  // namespace
+
+bool seed_oblivious(const Kernel& k, std::vector<bool>* tainted) {
+    Taint T;
+    T.tv.assign(k.vars.size(), false);
+    for (const ArrayDecl& a : k.arrays)
+        if (a.space == PRIVATE) T.ok = false;
+    while (T.prop(k.body)) {
+    }
+    T.check(k.body);
+    if (tainted) *tainted = T.tv;
+    return T.ok;
+}
 
 std::string generate_cuda(const Kernel& k, const CodegenOptions& opt) {
     Gen g(k, opt);

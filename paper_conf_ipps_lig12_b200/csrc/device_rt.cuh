@@ -144,6 +144,7 @@ struct PgT {        // hot per-emulated-thread state (kept in registers)
     u32 l0cell, l0val, l0site;  // write-log entry 0 (registers; entries 1.. live in PgCold)
     u32 fuel;
     u32 sg;         // byte offset of this instance's shared region in pg_dsmem
+    u32 nsv;        // multi-seed lanes: seeds of this lane's group (<= PG_MS)
     u64 seed;
     u32* arena;     // this instance's kernel arena
     const u32* input;
@@ -178,7 +179,17 @@ __device__ __noinline__ u32 pg_event(PgCold& c, u32 evm, u32 kind, u32 round, u3
     c.ecnt[kind] = has ? c.ecnt[kind] + 1u : 1u;
     return 1u << kind;
 }
+#ifndef PG_MS
+#define PG_MS 1
+#endif
+#define PG_S_LOOP _Pragma("unroll") for (u32 _s = 0; _s < (u32)PG_MS; _s++)
+#if PG_MS > 1
+// multi-seed lanes (optimistic pass only): an event flags the lane's instances, whose
+// records the exact re-run then produces seed by seed
+#define PG_EVENT(t, c, ...) ((t).fl = 1u)
+#else
 #define PG_EVENT(t, c, ...) ((t).evm |= pg_event((c), (t).evm, __VA_ARGS__))
+#endif
 
 // stamps: step (20 bits, >= 1) and block-local tid (12 bits)
 __device__ __forceinline__ u32 pg_stamp_min(const PgC& C, const PgT& t) { return C.smin | t.tlin; }
@@ -507,6 +518,147 @@ __device__ __forceinline__ void pg_st_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32
     pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
 #endif
 }
+
+#if PG_MS > 1
+// ------------------------------------------------------------------ multi-seed lanes
+// Optimistic pass of a seed-oblivious kernel (codegen seed_oblivious): the PG_MS seeds of
+// a group take the same accesses, so one lane evaluates the address, guard, stamp and
+// race logic once and carries PG_MS values.  Shared values are laid out [cell][seed]
+// (one 128-bit access for PG_MS = 4); stamps are per cell as before.  Anything that
+// would be an event (OOB, UNINIT, LIMIT, a race) flags the group's instances, which the
+// exact single-seed re-run then evaluates and records.
+__device__ __forceinline__ void pg_vld(const u32* p, u32 (&v)[PG_MS]) {
+#if PG_MS == 4
+    const uint4 q = *(const uint4*)p;
+    v[0] = q.x; v[1] = q.y; v[2] = q.z; v[3] = q.w;
+#elif PG_MS == 2
+    const uint2 q = *(const uint2*)p;
+    v[0] = q.x; v[1] = q.y;
+#else
+    PG_S_LOOP v[_s] = p[_s];
+#endif
+}
+__device__ __forceinline__ void pg_vst(u32* p, const u32 (&v)[PG_MS]) {
+#if PG_MS == 4
+    *(uint4*)p = make_uint4(v[0], v[1], v[2], v[3]);
+#elif PG_MS == 2
+    *(uint2*)p = make_uint2(v[0], v[1]);
+#else
+    PG_S_LOOP p[_s] = v[_s];
+#endif
+}
+template <int A, bool RD, bool LOG>
+__device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
+                                            u32 (&v)[PG_MS]) {
+    const u32 inb = flat < PG_SH(A, size);
+    u32 own = 0u;
+    if (pe & inb) {
+        if (RD && PG_T > 1u) {
+            const u32 so = C.par * PG_SH(A, size) + flat;
+            atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + so, C.smin | t.tlin);
+            atomicMax(pg_sh(t, PG_SH(A, s_rmax)) + so, C.smax | t.tlin);
+        }
+        own = pg_sh(t, PG_SH(A, s_own))[flat];
+        pg_vld(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
+    } else {
+        PG_S_LOOP v[_s] = 0u;
+    }
+    t.fl |= pe & ((inb ^ 1u) | (u32)(own >= C.uthr));   // OOB / never written (X5, X6)
+}
+template <int A, bool RDA = false>
+__device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat,
+                                            const u32 (&val)[PG_MS], u32 site) {
+    if (!pe) return;
+    if (flat >= PG_SH(A, size)) {
+        t.fl = 1u;
+        return;
+    }
+    u32* own = pg_sh(t, PG_SH(A, s_own)) + flat;
+    const u32 me = C.smin | t.tlin;
+    if (PG_T > 1u) {
+        const u32 old = atomicMin(own, me);
+        t.fl |= (old ^ me) - 1u < 0xFFFu;   // another writer's stamp of this round (WW)
+        if (RDA) pg_flog(t, c, ((u32)A << 24) | flat);
+    } else {
+        *own = me;
+    }
+    pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, val);
+    pg_fcount(t);
+}
+// global arrays: per-seed arenas (values, last writer and the XB block marks are read per
+// instance by K2b/K3); owner and reader stamps agree across the seeds and live in the
+// group's first arena only
+template <int A>
+__device__ __forceinline__ void pg_xb_mark_ms(const PgT& t, u32 flat) {
+    if (pg_sL.nblocks > 1u) {
+        const u64 st = pg_sL.arena_stride;
+        PG_S_LOOP {
+            if (_s < t.nsv) {
+                atomicMin(t.arena + _s * st + PG_ARR(A).off_xf + flat, t.blk + 1u);
+                atomicMax(t.arena + _s * st + PG_ARR(A).off_xl + flat, t.blk + 1u);
+            }
+        }
+    }
+}
+template <int A, bool RD, bool LOG>
+__device__ __forceinline__ void pg_ld_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
+                                            u32 (&v)[PG_MS]) {
+    PG_S_LOOP v[_s] = 0u;
+    if (!pe) return;
+    if (flat >= PG_ARR(A).size) {
+        t.fl = 1u;
+        return;
+    }
+    pg_xb_mark_ms<A>(t, flat);
+    if (RD && PG_T > 1u) {
+        const u64 so = (u64)C.par * PG_ARR(A).size + flat;
+        atomicMin(t.arena + PG_ARR(A).off_rmin + so, C.smin | t.tlin);
+        atomicMax(t.arena + PG_ARR(A).off_rmax + so, C.smax | t.tlin);
+    }
+    const u64 st = pg_sL.arena_stride;
+    PG_S_LOOP if (_s < t.nsv) v[_s] = t.arena[_s * st + PG_ARR(A).off_val + flat];
+}
+template <int A, bool RDA = false>
+__device__ __forceinline__ void pg_st_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat,
+                                            const u32 (&val)[PG_MS], u32 site) {
+    if (!pe) return;
+    if (flat >= PG_ARR(A).size) {
+        t.fl = 1u;
+        return;
+    }
+    pg_xb_mark_ms<A>(t, flat);
+    u32* own = t.arena + PG_ARR(A).off_own + flat;
+    const u32 me = C.smin | t.tlin;
+    if (PG_T > 1u) {
+        const u32 old = atomicMin(own, me);
+        t.fl |= (old ^ me) - 1u < 0xFFFu;
+        if (RDA) pg_flog(t, c, ((u32)A << 24) | flat);
+    } else {
+        *own = me;
+    }
+    const u64 st = pg_sL.arena_stride;
+    PG_S_LOOP {
+        if (_s < t.nsv) {
+            t.arena[_s * st + PG_ARR(A).off_val + flat] = val[_s];
+            t.arena[_s * st + PG_ARR(A).off_lw + flat] = t.gtid + 1u;
+        }
+    }
+    pg_fcount(t);
+}
+template <int A>
+__device__ __forceinline__ void pg_ld_gi_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
+                                            u32 (&v)[PG_MS]) {
+    PG_S_LOOP v[_s] = 0u;
+    if (!pe) return;
+    if (flat >= PG_ARR(A).size) {
+        t.fl = 1u;
+        return;
+    }
+    const u32* p = t.input + PG_ARR(A).off_in + flat;
+    const u64 st = pg_sL.input_stride;
+    PG_S_LOOP v[_s] = __ldg(p + (u64)min(_s, t.nsv - 1u) * st);
+}
+#endif
 
 // XB bookkeeping (X4): first and last block that accessed a global cell.  Kept
 // whenever the launch has more than one block (it also decides whether the
@@ -1052,6 +1204,8 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     const u32 inst_ok = lane_ok && g < G && (P.seq != 2u || P.xb_flag[pg_sW.inst0 + g / GB] != 0u);
     const u32 gc = inst_ok ? g : 0u;
     const u32 ms = gc / GB, bs = gc % GB;
+    const u32 sb = ms * PG_MS;   // the group's first seed within the item (multi-seed lanes: PG_MS seeds)
+    const u32 nsv = PG_MS > 1 ? min((u32)PG_MS, pg_sW.nseeds - min(sb, pg_sW.nseeds)) : 1u;
     typename K::Frame F[PG_VMAX];
     PgT T[PG_VMAX];
     PgCold Cd[PG_VMAX];
@@ -1067,9 +1221,10 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         t.tid[0] = t.tlin % PG_BDIM0;
         t.tid[1] = (t.tlin / PG_BDIM0) % PG_BDIM1;
         t.tid[2] = t.tlin / (PG_BDIM0 * PG_BDIM1);
-        t.seed = P.seed_base + (u64)(pg_sW.seed_j0 + ms * pg_sW.seed_jstep);
-        t.arena = P.arena + pg_sW.arena_off + (u64)ms * pg_sL.arena_stride;
-        t.input = P.input + pg_sW.input_off + (u64)ms * pg_sL.input_stride;
+        t.seed = P.seed_base + (u64)(pg_sW.seed_j0 + sb * pg_sW.seed_jstep);
+        t.arena = P.arena + pg_sW.arena_off + (u64)sb * pg_sL.arena_stride;
+        t.input = P.input + pg_sW.input_off + (u64)sb * pg_sL.input_stride;
+        t.nsv = nsv;
         t.sg = gc * gbytes;
         t.l0cell = t.l0val = t.l0site = 0u;
         t.evm = 0u;
@@ -1256,7 +1411,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
-                pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)ms * pg_sW.slot_step,
+                pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)sb * pg_sW.slot_step,
                              s_flush);
             }
         }
@@ -1269,21 +1424,26 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             if (v >= V) break;
             fl |= T[v].fl;
         }
-        if (fl && inst_ok) P.xb_flag[pg_sW.inst0 + ms] = 1u;
+        if (fl && inst_ok)
+            for (u32 i = 0; i < nsv; i++) P.xb_flag[pg_sW.inst0 + sb + i] = 1u;
     }
 #endif
     // instances (X19) per batch-local instance (a re-run replaces its instance's count):
     // one atomic per warp when the warp's groups belong to one instance (block-major packing)
     if (P.count_inst) {
         u64 x = (inst_ok && tl0 == 0u) ? inst : 0ull;
-        const u32 key = x ? pg_sW.inst0 + ms : PG_NEVER;
+        const u32 key = x ? pg_sW.inst0 + sb : PG_NEVER;
         const u32 k0 = __reduce_min_sync(PG_FULL, key);
         if (__all_sync(PG_FULL, key == PG_NEVER || key == k0)) {
 #pragma unroll
             for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(PG_FULL, x, o);
-            if (lane == 0u && x) atomicAdd(&P.inst_cnt[k0], x);
+            if (lane == 0u && x) {
+                // (multi-seed lanes: every seed of the group ran the same rounds)
+                const u32 n0 = PG_MS > 1 ? min((u32)PG_MS, pg_sW.nseeds - (k0 - pg_sW.inst0)) : 1u;
+                for (u32 i = 0; i < n0; i++) atomicAdd(&P.inst_cnt[k0 + i], x);
+            }
         } else if (x) {
-            atomicAdd(&P.inst_cnt[key], x);
+            for (u32 i = 0; i < nsv; i++) atomicAdd(&P.inst_cnt[key + i], x);
         }
     }
 #if PG_BANKCHK || PG_COALCHK

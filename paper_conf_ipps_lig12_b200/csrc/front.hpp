@@ -126,7 +126,14 @@ struct CodegenOptions {
     uint32_t bank_model = 0;
     uint32_t wmax = 32;
     bool fast = false;   // optimistic pass: in-place commits, race detection only
+    uint32_t ms = 1;     // optimistic pass of a seed-oblivious kernel: seeds per lane
 };
 std::string generate_cuda(const Kernel& k, const CodegenOptions& opt);
+
+// Multi-seed lanes: true when no address, access guard, branch or loop condition of the
+// kernel depends on array contents (and it has no private arrays), so every seed of a
+// launch performs the same accesses in the same rounds and only the values differ.
+// tainted[v]: variable v may hold an input-dependent value (one copy per seed).
+bool seed_oblivious(const Kernel& k, std::vector<bool>* tainted = nullptr);
 
 }  // namespace pgf
