@@ -721,12 +721,13 @@ struct Gen {
         }
         o << "      default: break;\n    }\n  }\n";
         o << "  static __device__ __forceinline__ void check_one(const PgC& C, PgT& t, PgCold& c, u32 cell, "
-             "u32 val, u32 site) {\n";
+             "pg_lv_t val, u32 site) {\n";
         o << "    const u32 flat = cell & 0xFFFFFFu;\n    switch (cell >> 24) {\n";
         for (size_t a = 0; a < K.arrays.size(); a++) {
             const ArrayDecl& A = K.arrays[a];
             if (!A.written || A.space == PRIVATE) continue;
-            o << "      case " << a << ": pg_check_" << (A.space == SHARED ? "sh" : "gt") << "<" << a << ", "
+            o << "      case " << a << ": pg_check_" << (A.space == SHARED ? "sh" : "gt") << (ms() && !O.fast ? "_ms" : "")
+              << "<" << a << ", "
               << (reader_tracked((int)a) ? "true" : "false") << ">(C, t, c, flat, val, site); break;\n";
         }
         o << "      default: break;\n    }\n  }\n";

@@ -22,6 +22,17 @@
 
 #include "pg_layout.h"
 
+// multi-seed lanes: PG_MS seeds per lane; PG_MSX: the exact protocol's
+// multi-seed variant (the re-run of instances the multi-seed optimistic pass flagged)
+#ifndef PG_MS
+#define PG_MS 1
+#endif
+#ifndef PG_FAST
+#define PG_FAST 0
+#endif
+#define PG_MSX (PG_MS > 1 && !PG_FAST)
+#define PG_S_LOOP _Pragma("unroll") for (u32 _s = 0; _s < (u32)PG_MS; _s++)
+
 // ------------------------------------------------------------------ arithmetic (X2)
 #define PG_MASK (PG_BITS >= 32 ? 0xFFFFFFFFu : ((1u << (PG_BITS & 31)) - 1u))
 __device__ __forceinline__ u32 pg_m(u32 v) { return PG_BITS >= 32 ? v : (v & PG_MASK); }
@@ -142,6 +153,9 @@ struct PgT {        // hot per-emulated-thread state (kept in registers)
     u32 evm;        // kinds with a recorded event (bit k: PgCold::ecnt[k] / ebest[k] are valid)
     u32 fl;         // PG_FAST: this thread saw a possible race / write-log overflow (instance re-run exactly)
     u32 l0cell, l0val, l0site;  // write-log entry 0 (registers; entries 1.. live in PgCold)
+#if PG_MSX
+    u32 l0v[PG_MS];             // (multi-seed exact pass: entry 0's value per seed)
+#endif
     u32 fuel;
     u32 sg;         // byte offset of this instance's shared region in pg_dsmem
     u32 nsv;        // multi-seed lanes: seeds of this lane's group (<= PG_MS)
@@ -150,12 +164,22 @@ struct PgT {        // hot per-emulated-thread state (kept in registers)
     const u32* input;
 };
 
+#if PG_MSX
+typedef const u32* pg_lv_t;   // a write-log value: one word per seed
+#else
+typedef u32 pg_lv_t;
+#endif
 struct PgCold {     // per-emulated-thread state that lives in local memory
     u32 lcell[PG_WMAX];   // write log entries 1.. (X3): cell id = array << 24 | flat
     u32 lval[PG_WMAX];
     u16 lsite[PG_WMAX];
     u32 ecnt[PG_NK];      // events per kind       (valid where PgT::evm has bit k: never initialised,
     u32 ebest[PG_NK][8];  // minimum event per kind  so threads without events touch no local memory) (X16)
+#if PG_MSX
+    u32 lvs[PG_WMAX][PG_MS];   // (see pg_lv_t)     // write-log values per seed (entries 1..)
+    u32 ebv[PG_NK][PG_MS][2];    // per seed: (val_a, val_b) of the minimum event; fields 0..5 of
+                                 // ebest are seed-independent (same accesses in every seed)
+#endif
 };
 
 __device__ __forceinline__ bool pg_lex_less(const u32* a, const u32* b) {
@@ -179,13 +203,20 @@ __device__ __noinline__ u32 pg_event(PgCold& c, u32 evm, u32 kind, u32 round, u3
     c.ecnt[kind] = has ? c.ecnt[kind] + 1u : 1u;
     return 1u << kind;
 }
-#ifndef PG_MS
-#define PG_MS 1
-#endif
-#define PG_S_LOOP _Pragma("unroll") for (u32 _s = 0; _s < (u32)PG_MS; _s++)
-#if PG_MS > 1
-// multi-seed lanes (optimistic pass only): an event flags the lane's instances, whose
-// records the exact re-run then produces seed by seed
+#if PG_MSX
+// multi-seed exact pass: events carry one value per seed (scalar values broadcast)
+__device__ __noinline__ u32 pg_event_ms(PgCold& c, u32 evm, u32 kind, u32 round, u32 arr, u32 addr, u32 ta,
+                                        u32 tb, u32 site, const u32* va, u32 vb);
+__device__ __forceinline__ u32 pg_event_msc(PgCold& c, u32 evm, u32 kind, u32 round, u32 arr, u32 addr, u32 ta,
+                                            u32 tb, u32 site, u32 va, u32 vb) {
+    u32 v[PG_MS];
+    PG_S_LOOP v[_s] = va;
+    return pg_event_ms(c, evm, kind, round, arr, addr, ta, tb, site, v, vb);
+}
+#define PG_EVENT(t, c, ...) ((t).evm |= pg_event_msc((c), (t).evm, __VA_ARGS__))
+#elif PG_MS > 1
+// multi-seed optimistic pass: an event flags the lane's instances, whose records the
+// exact re-run then produces
 #define PG_EVENT(t, c, ...) ((t).fl = 1u)
 #else
 #define PG_EVENT(t, c, ...) ((t).evm |= pg_event((c), (t).evm, __VA_ARGS__))
@@ -553,6 +584,7 @@ __device__ __forceinline__ void pg_vst(u32* p, const u32 (&v)[PG_MS]) {
     PG_S_LOOP p[_s] = v[_s];
 #endif
 }
+#if PG_FAST
 template <int A, bool RD, bool LOG>
 __device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
                                             u32 (&v)[PG_MS]) {
@@ -664,6 +696,261 @@ __device__ __forceinline__ void pg_ld_gi_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     const u64 st = pg_sL.input_stride;
     PG_S_LOOP v[_s] = __ldg(p + (u64)min(_s, t.nsv - 1u) * st);
 }
+#else   // PG_MSX: the exact protocol, PG_MS seeds per lane
+// Per seed: write-log values, committed values, poison values and the events' value
+// fields; once per cell: claims, owner / race stamps and the race decision.
+__device__ __forceinline__ u64 pg_seed_of(const PgT& t, u32 s) { return t.seed + (u64)s * pg_sW.seed_jstep; }
+__device__ __noinline__ u32 pg_event_ms(PgCold& c, u32 evm, u32 kind, u32 round, u32 arr, u32 addr, u32 ta,
+                                        u32 tb, u32 site, const u32* va, u32 vb) {
+    const u32 e[6] = {round, arr, addr, ta, tb, site};
+    const u32 has = (evm >> kind) & 1u;
+    int cmp = -1;
+    if (has) {
+        cmp = 0;
+        for (int i = 0; i < 6 && cmp == 0; i++)
+            if (e[i] != c.ebest[kind][i]) cmp = e[i] < c.ebest[kind][i] ? -1 : 1;
+    }
+    if (cmp < 0) {
+        for (int i = 0; i < 6; i++) c.ebest[kind][i] = e[i];
+        PG_S_LOOP { c.ebv[kind][_s][0] = va[_s]; c.ebv[kind][_s][1] = vb; }
+    } else if (cmp == 0) {   // same access: the per-seed values decide (X16 lexicographic order)
+        PG_S_LOOP {
+            if (va[_s] < c.ebv[kind][_s][0] || (va[_s] == c.ebv[kind][_s][0] && vb < c.ebv[kind][_s][1])) {
+                c.ebv[kind][_s][0] = va[_s];
+                c.ebv[kind][_s][1] = vb;
+            }
+        }
+    }
+    c.ecnt[kind] = has ? c.ecnt[kind] + 1u : 1u;
+    return 1u << kind;
+}
+__device__ __forceinline__ u32 pg_log_find_ms(const PgT& t, const PgCold& c, u32 cell, u32 (&v)[PG_MS]) {
+    if (t.nlog == 0u) return 0u;
+    if (t.l0cell == cell) {
+        PG_S_LOOP v[_s] = t.l0v[_s];
+        return 1u;
+    }
+    for (u32 i = 1; i < t.nlog; i++)
+        if (c.lcell[i] == cell) {
+            PG_S_LOOP v[_s] = c.lvs[i][_s];
+            return 1u;
+        }
+    return 0u;
+}
+__device__ __noinline__ u32 pg_log_write_slow_ms(u32 nlog, PgCold& c, u32 cell, const u32* val, u32 site) {
+    for (u32 i = 1; i < nlog; i++) {
+        if (c.lcell[i] == cell) {
+            PG_S_LOOP c.lvs[i][_s] = val[_s];
+            c.lsite[i] = (u16)site;
+            return nlog;
+        }
+    }
+    if (nlog >= PG_WMAX) return PG_NEVER;
+    c.lcell[nlog] = cell;
+    PG_S_LOOP c.lvs[nlog][_s] = val[_s];
+    c.lsite[nlog] = (u16)site;
+    return nlog + 1u;
+}
+__device__ __forceinline__ void pg_log_write_ms(PgC& C, PgT& t, PgCold& c, u32 cell, const u32 (&val)[PG_MS],
+                                                u32 site, u32 rec, u32 flat) {
+    if (t.nlog == 0u) {
+        t.l0cell = cell;
+        PG_S_LOOP t.l0v[_s] = val[_s];
+        t.l0site = site;
+        t.nlog = 1u;
+    } else if (t.l0cell == cell) {
+        PG_S_LOOP t.l0v[_s] = val[_s];
+        t.l0site = site;
+    } else {
+        const u32 n = pg_log_write_slow_ms(t.nlog, c, cell, val, site);
+        if (n == PG_NEVER) PG_EVENT(t, c, PGK_LIMIT, C.round, rec, flat, t.gtid, PG_NEVER, site, 1, 0);
+        else t.nlog = n;
+    }
+}
+template <int A, bool RD, bool LOG>
+__device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
+                                            u32 (&v)[PG_MS]) {
+    PG_S_LOOP v[_s] = 0u;
+    if (!pe) return;
+    const u32 rec = PG_ARR(A).rec_id;
+    if (flat >= PG_SH(A, size)) {
+        PG_S_LOOP v[_s] = pg_m(pg_rand32(pg_seed_of(t, _s), 0x8000u + (rec - 0x100u), ((u64)t.blk << 20) + flat));
+#if PG_OOBCHK
+        t.evm |= pg_event_ms(c, t.evm, PGK_OOB, C.round, rec, flat, t.gtid, PG_NEVER, site, v, 0);
+#endif
+        return;
+    }
+#if PG_RACECHK
+    if (RD && PG_T > 1u) {
+        atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + flat, pg_stamp_min(C, t));
+        atomicMax(pg_sh(t, PG_SH(A, s_rmax)) + flat, pg_stamp_max(C, t));
+    }
+#endif
+    if (LOG && pg_log_find_ms(t, c, ((u32)A << 24) | flat, v)) return;
+    const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
+    if (own >= C.uthr) {  // never written in this block (X6)
+        PG_S_LOOP v[_s] = pg_m(pg_rand32(pg_seed_of(t, _s), 0x8000u + (rec - 0x100u), ((u64)t.blk << 20) + flat));
+#if PG_OOBCHK
+        t.evm |= pg_event_ms(c, t.evm, PGK_UNINIT, C.round, rec, flat, t.gtid, PG_NEVER, site, v, 0);
+#endif
+        return;
+    }
+    pg_vld(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
+}
+template <int A, bool RDA = false>
+__device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat,
+                                            const u32 (&val)[PG_MS], u32 site) {
+    if (!pe) return;
+    if (flat >= PG_SH(A, size)) {
+#if PG_OOBCHK
+        t.evm |= pg_event_ms(c, t.evm, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, val, 1);
+#endif
+        return;
+    }
+    pg_log_write_ms(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+}
+template <int A>
+__device__ __forceinline__ void pg_xb_mark_ms(const PgT& t, u32 flat) {
+    if (pg_sL.nblocks > 1u) {
+        const u64 st = pg_sL.arena_stride;
+        PG_S_LOOP {
+            if (_s < t.nsv) {
+                atomicMin(t.arena + _s * st + PG_ARR(A).off_xf + flat, t.blk + 1u);
+                atomicMax(t.arena + _s * st + PG_ARR(A).off_xl + flat, t.blk + 1u);
+            }
+        }
+    }
+}
+template <int A, bool RD, bool LOG>
+__device__ __forceinline__ void pg_ld_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
+                                            u32 (&v)[PG_MS]) {
+    PG_S_LOOP v[_s] = 0u;
+    if (!pe) return;
+    if (flat >= PG_ARR(A).size) {
+        PG_S_LOOP v[_s] = pg_m(pg_rand32(pg_seed_of(t, _s), PG_ARR(A).gid, flat));
+#if PG_OOBCHK
+        t.evm |= pg_event_ms(c, t.evm, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, v, 0);
+#endif
+        return;
+    }
+    pg_xb_mark_ms<A>(t, flat);
+#if PG_RACECHK
+    if (RD && PG_T > 1u) {
+        atomicMin(t.arena + PG_ARR(A).off_rmin + flat, pg_stamp_min(C, t));
+        atomicMax(t.arena + PG_ARR(A).off_rmax + flat, pg_stamp_max(C, t));
+    }
+#endif
+    if (LOG && pg_log_find_ms(t, c, ((u32)A << 24) | flat, v)) return;
+    const u64 st = pg_sL.arena_stride;
+    PG_S_LOOP if (_s < t.nsv) v[_s] = t.arena[_s * st + PG_ARR(A).off_val + flat];
+}
+template <int A, bool RDA = false>
+__device__ __forceinline__ void pg_st_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat,
+                                            const u32 (&val)[PG_MS], u32 site) {
+    if (!pe) return;
+    if (flat >= PG_ARR(A).size) {
+#if PG_OOBCHK
+        t.evm |= pg_event_ms(c, t.evm, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, val, 1);
+#endif
+        return;
+    }
+    pg_xb_mark_ms<A>(t, flat);
+    pg_log_write_ms(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+}
+template <int A>
+__device__ __forceinline__ void pg_ld_gi_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
+                                            u32 (&v)[PG_MS]) {
+    PG_S_LOOP v[_s] = 0u;
+    if (!pe) return;
+    if (flat >= PG_ARR(A).size) {
+        PG_S_LOOP v[_s] = pg_m(pg_rand32(pg_seed_of(t, _s), PG_ARR(A).gid, flat));
+#if PG_OOBCHK
+        t.evm |= pg_event_ms(c, t.evm, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, v, 0);
+#endif
+        return;
+    }
+    const u32* p = t.input + PG_ARR(A).off_in + flat;
+    const u64 st = pg_sL.input_stride;
+    PG_S_LOOP v[_s] = __ldg(p + (u64)min(_s, t.nsv - 1u) * st);
+}
+// round end of the exact protocol: the owner commits every seed's value; race decisions
+// are per cell, their records carry each seed's value
+__device__ __noinline__ u32 pg_race_check_ms(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 evm,
+                                             const u32* val, u32 site, u32 rec, u32 flat, u32 own, u32 wmax,
+                                             u32 has_readers, u32 rmin, u32 rmax) {
+    const u32 base = gtid - tlin;
+    const u32 w0 = own & 0xFFFu, w1 = wmax & 0xFFFu;
+    if (w1 != w0 && tlin == w0) evm |= pg_event_ms(c, evm, PGK_WW, round, rec, flat, gtid, base + w1, site, val, 0);
+    if (has_readers && (rmax >> 12) == step) {
+        const u32 r0 = rmin & 0xFFFu, r1 = rmax & 0xFFFu;
+        if (!(r0 == r1 && w0 == w1 && r0 == w0)) {
+            u32 ta, tb;
+            if (r0 != w0) { ta = w0; tb = r0; }
+            else if (r1 != w0) { ta = w0; tb = r1; }
+            else { ta = w1; tb = r0; }
+            if (tlin == ta) evm |= pg_event_ms(c, evm, PGK_RW, round, rec, flat, base + ta, base + tb, site, val, 0);
+        }
+    }
+    return evm;
+}
+template <int A, bool RD>
+__device__ __forceinline__ void pg_check_sh_ms(const PgC& C, PgT& t, PgCold& c, u32 flat, const u32* val, u32 site) {
+    u32 v[PG_MS];
+    PG_S_LOOP v[_s] = val[_s];
+    if (PG_T == 1u) {
+        pg_sh(t, PG_SH(A, s_own))[flat] = pg_stamp_min(C, t);
+        pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
+        return;
+    }
+    const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
+    if (own == pg_stamp_min(C, t)) pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
+#if PG_RACECHK
+    if (PG_T > 1u) {
+        const u32 wmax = pg_sh(t, PG_SH(A, s_wmax))[flat];
+        const u32 rmin = RD ? pg_sh(t, PG_SH(A, s_rmin))[flat] : 0u;
+        const u32 rmax = RD ? pg_sh(t, PG_SH(A, s_rmax))[flat] : 0u;
+        if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
+            (RD && (rmax >> 12) == C.step && (((rmin ^ own) | (rmax ^ own)) & 0xFFFu)))
+            t.evm = pg_race_check_ms(C.round, C.step, t.tlin, t.gtid, c, t.evm, val, site, PG_ARR(A).rec_id, flat,
+                                     own, wmax, RD, rmin, rmax);
+    }
+#endif
+}
+template <int A, bool RD>
+__device__ __forceinline__ void pg_check_gt_ms(const PgC& C, PgT& t, PgCold& c, u32 flat, const u32* val, u32 site) {
+    const u64 st = pg_sL.arena_stride;
+    if (PG_T == 1u) {
+        t.arena[PG_ARR(A).off_own + flat] = pg_stamp_min(C, t);
+        PG_S_LOOP {
+            if (_s < t.nsv) {
+                t.arena[_s * st + PG_ARR(A).off_val + flat] = val[_s];
+                t.arena[_s * st + PG_ARR(A).off_lw + flat] = t.gtid + 1u;
+            }
+        }
+        return;
+    }
+    const u32 own = t.arena[PG_ARR(A).off_own + flat];
+    if (own == pg_stamp_min(C, t)) {
+        PG_S_LOOP {
+            if (_s < t.nsv) {
+                t.arena[_s * st + PG_ARR(A).off_val + flat] = val[_s];
+                t.arena[_s * st + PG_ARR(A).off_lw + flat] = t.gtid + 1u;
+            }
+        }
+    }
+#if PG_RACECHK
+    if (PG_T > 1u) {
+        const u32 wmax = t.arena[PG_ARR(A).off_wmax + flat];
+        const u32 rmin = RD ? t.arena[PG_ARR(A).off_rmin + flat] : 0u;
+        const u32 rmax = RD ? t.arena[PG_ARR(A).off_rmax + flat] : 0u;
+        if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
+            (RD && (rmax >> 12) == C.step && (((rmin ^ own) | (rmax ^ own)) & 0xFFFu)))
+            t.evm = pg_race_check_ms(C.round, C.step, t.tlin, t.gtid, c, t.evm, val, site, PG_ARR(A).rec_id, flat,
+                                     own, wmax, RD, rmin, rmax);
+    }
+#endif
+}
+#endif   // PG_FAST
 #endif
 
 // XB bookkeeping (X4): first and last block that accessed a global cell.  Kept
@@ -896,8 +1183,13 @@ __device__ __forceinline__ void pg_claim_all(const PgC& C, const PgT& t, const P
 template <class K>
 __device__ __forceinline__ void pg_check_all(const PgC& C, PgT& t, PgCold& c) {
     if (t.nlog == 0u) return;
+#if PG_MSX
+    K::check_one(C, t, c, t.l0cell, t.l0v, t.l0site);
+    for (u32 i = 1; i < t.nlog; i++) K::check_one(C, t, c, c.lcell[i], c.lvs[i], c.lsite[i]);
+#else
     K::check_one(C, t, c, t.l0cell, t.l0val, t.l0site);
     for (u32 i = 1; i < t.nlog; i++) K::check_one(C, t, c, c.lcell[i], c.lval[i], c.lsite[i]);
+#endif
 }
 
 #if PG_LOCKSTEP
@@ -1029,7 +1321,7 @@ __device__ __noinline__ void pg_slot_update(PgSlot* s, u32 cnt, const u32* best)
 }
 
 __device__ __noinline__ void pg_flush_cta(const PgParams& P, u32 lane, u32 warp, PgCold& c, u32 evm, u32 valid,
-                                          u64 slot0, PgFlushEntry* sh /* [32] in shared memory */) {
+                                          u64 slot0, PgFlushEntry* sh /* [32] in shared memory */, u32 seed_s = 0) {
     const u32 nwarps = blockDim.x >> 5;
     const u32 warp_evm = __reduce_or_sync(PG_FULL, valid ? evm : 0u);
     for (u32 k = 0; k < PG_NK; k++) {
@@ -1045,6 +1337,10 @@ __device__ __noinline__ void pg_flush_cta(const PgParams& P, u32 lane, u32 warp,
             u32 f_in[8];
 #pragma unroll
             for (int i = 0; i < 8; i++) f_in[i] = pending ? c.ebest[k][i] : PG_NEVER;
+#if PG_MSX
+            f_in[6] = pending ? c.ebv[k][seed_s][0] : PG_NEVER;   // (multi-seed exact pass: this seed's values)
+            f_in[7] = pending ? c.ebv[k][seed_s][1] : PG_NEVER;
+#endif
             pg_warp_merge(pending, slot0, pending ? c.ecnt[k] : 0u, f_in, lane, leader, key, cnt, best, members);
             if (lane == leader) {
                 if (first) {   // the common case: one instance per warp -> deposit for the CTA merge
@@ -1207,7 +1503,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         ekey = 0u;
     }
     // (exact re-run, P.seq == 2: only the instances the optimistic pass flagged)
-    const u32 inst_ok = lane_ok && g < G && (P.seq != 2u || P.xb_flag[pg_sW.inst0 + g / GB] != 0u);
+    const u32 inst_ok = lane_ok && g < G && (P.seq != 2u || P.xb_flag[pg_sW.inst0 + (g / GB) * PG_MS] != 0u);
     const u32 gc = inst_ok ? g : 0u;
     const u32 ms = gc / GB, bs = gc % GB;
     const u32 sb = ms * PG_MS;   // the group's first seed within the item (multi-seed lanes: PG_MS seeds)
@@ -1417,8 +1713,14 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
+#if PG_MSX
+                for (u32 q = 0; q < PG_MS; q++)   // one slot per seed of the group
+                    pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_ && q < nsv,
+                                 pg_sW.slot0 + (u64)(sb + q) * pg_sW.slot_step, s_flush, q);
+#else
                 pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)sb * pg_sW.slot_step,
                              s_flush);
+#endif
             }
         }
     }
