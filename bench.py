@@ -95,6 +95,20 @@ class Clocks:
             if len(parts) >= 7:
                 self.rows.append(parts)
 
+    def wait_first(self, timeout=5.0):
+        """Block until nvidia-smi delivers its first sample (its start-up takes longer than a
+        short timed region), so every later sample falls inside the region."""
+        t0 = time.time()
+        while self.proc is not None and not self.rows and time.time() - t0 < timeout:
+            time.sleep(0.01)
+        self.skip = len(self.rows)
+
+    def wait_sample(self, timeout=1.0):
+        """Block until at least one sample was taken after wait_first (the region's)."""
+        t0 = time.time()
+        while self.proc is not None and len(self.rows) <= getattr(self, "skip", 0) and time.time() - t0 < timeout:
+            time.sleep(0.01)
+
     def stop(self):
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
@@ -105,12 +119,13 @@ class Clocks:
             self.proc.kill()
         if self.thread:
             self.thread.join(timeout=2)
-        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        rows = self.rows[getattr(self, "skip", 0):]   # samples taken inside the timed region
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() == "active"})
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[3 + i].lower() == "active"})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+                "reasons": reasons, "samples": len(rows)}
 
 
 def dist_env():
@@ -198,11 +213,11 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="pgvc", choices=["pgvc", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--ref-log-n", type=int, default=14)
+    ap.add_argument("--ref-log-n", type=int, default=13, help="reference arm: C2 sample N <= 2^k per step")
     ap.add_argument("--ref-seeds", type=int, default=0, help="0: one seed per host core")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + 1 step, no JSON (for ncu launch lists)")
     ap.add_argument("--diag", action="store_true", help="print per-step enqueue / device / per-check times")
@@ -301,6 +316,7 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     clocks.start()
+    clocks.wait_first()
     evs, all_runs = [], []
     for k in range(args.steps):
         with torch.cuda.stream(stream):
@@ -310,6 +326,7 @@ def main():
         all_runs.append(step(keys[k], cnts[k]))
         e1.record(stream)
         evs.append((e0, e1))
+    clocks.wait_sample(timeout=2.0)   # (the enqueued steps are still running: a sample under load)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()

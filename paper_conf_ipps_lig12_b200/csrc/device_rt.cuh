@@ -1320,12 +1320,13 @@ __device__ __noinline__ void pg_slot_update(PgSlot* s, u32 cnt, const u32* best)
     atomicExch(&s->lock, 0u);
 }
 
+// kmask: the kinds some thread of the CTA recorded (CTA-uniform, from the caller)
 __device__ __noinline__ void pg_flush_cta(const PgParams& P, u32 lane, u32 warp, PgCold& c, u32 evm, u32 valid,
-                                          u64 slot0, PgFlushEntry* sh /* [32] in shared memory */, u32 seed_s = 0) {
+                                          u64 slot0, PgFlushEntry* sh /* [32] in shared memory */, u32 kmask,
+                                          u32 seed_s = 0) {
     const u32 nwarps = blockDim.x >> 5;
-    const u32 warp_evm = __reduce_or_sync(PG_FULL, valid ? evm : 0u);
     for (u32 k = 0; k < PG_NK; k++) {
-        if (!__syncthreads_or((int)((warp_evm >> k) & 1u))) continue;
+        if (!((kmask >> k) & 1u)) continue;
         if (lane == 0) sh[warp].slot = ~0ull;
         __syncwarp();
         u32 pending = valid && ((evm >> k) & 1u);
@@ -1709,17 +1710,27 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             if (v >= V) break;
             any_ev |= T[v].evm;
         }
-        if (__syncthreads_or((int)any_ev)) {
+        // the kinds recorded anywhere in the CTA: one barrier, then only those kinds are merged
+        __shared__ u32 s_kmask;
+        if (threadIdx.x == 0) s_kmask = 0u;
+        __syncthreads();
+        {
+            const u32 wm = __reduce_or_sync(PG_FULL, inst_ok ? any_ev : 0u);
+            if (lane == 0u && wm) atomicOr(&s_kmask, wm);
+        }
+        __syncthreads();
+        const u32 kmask = s_kmask;
+        if (kmask) {
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
 #if PG_MSX
                 for (u32 q = 0; q < PG_MS; q++)   // one slot per seed of the group
                     pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_ && q < nsv,
-                                 pg_sW.slot0 + (u64)(sb + q) * pg_sW.slot_step, s_flush, q);
+                                 pg_sW.slot0 + (u64)(sb + q) * pg_sW.slot_step, s_flush, kmask, q);
 #else
                 pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)sb * pg_sW.slot_step,
-                             s_flush);
+                             s_flush, kmask);
 #endif
             }
         }
@@ -1733,7 +1744,10 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             fl |= T[v].fl;
         }
         if (fl && inst_ok)
+        {
             for (u32 i = 0; i < nsv; i++) P.xb_flag[pg_sW.inst0 + sb + i] = 1u;
+            if (P.flag_any) *P.flag_any = 1u;
+        }
     }
 #endif
     // instances (X19) per batch-local instance (a re-run replaces its instance's count):
@@ -1772,6 +1786,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 // selection kernel listed: a pass with nothing to re-run costs one short launch.
 template <class K>
 __device__ __forceinline__ void pg_main(const PgParams& P) {
+    if (P.seq && P.flag_any && *(volatile const u32*)P.flag_any == 0u) return;   // nothing to re-run
     const bool listed = P.work_count != nullptr;
     const u32 n = listed ? *P.work_count : P.n_work ? P.n_work : blockIdx.x + 1u;
     for (u32 i = blockIdx.x; i < n; i += gridDim.x) {   // (one call site: one inlined copy)

@@ -51,7 +51,8 @@ __device__ __forceinline__ void pg_unit_words(const Units& u, u32 un, u32 n, u32
 // instances the optimistic pass flagged)
 __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ jobs, u32* arena_s, u32* arena_t,
                                                      u32* input, u64 seed_base, u32 mode, u32 range, u32 mask,
-                                                     const u32* flags) {
+                                                     const u32* flags, const u32* any) {
+    if (flags && !*any) return;   // re-initialisation with nothing flagged
     const PgFill f = jobs[blockIdx.y];
     u32* region = f.target == 0 ? arena_s : f.target == 1 ? arena_t : input;
     const Units u = pg_units(f.n);
@@ -148,7 +149,8 @@ __global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__
 
 // K2b: flag every instance in which some global cell written by the kernel was
 // accessed by two blocks (X4 XB) - the block-parallel pass is not exact there.
-__global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ jobs, const u32* arena, u32* flags) {
+__global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ jobs, const u32* arena, u32* flags,
+                                                    u32* any) {
     const PgXb j = jobs[blockIdx.y];
     if (j.n <= kSmallN) {   // a warp per instance
         const Units u = pg_units(j.n);
@@ -159,7 +161,10 @@ __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ job
                 const u32 xf = arena[j.xf + base + i], xl = arena[j.xl + base + i];
                 hit |= (xl != 0u && xf != xl && arena[j.lw + base + i] != 0u);
             }
-            if (__any_sync(0xffffffffu, hit) && u.tid == 0) flags[j.inst0 + inst] = 1u;
+            if (__any_sync(0xffffffffu, hit) && u.tid == 0) {
+                flags[j.inst0 + inst] = 1u;
+                *any = 1u;
+            }
         }
         return;
     }
@@ -173,7 +178,10 @@ __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ job
             const u32 xf = arena[j.xf + base + i], xl = arena[j.xl + base + i], lw = arena[j.lw + base + i];
             hit |= (xl != 0u) & (xf != xl) & (lw != 0u);
         }
-        if (__syncthreads_or((int)hit) && threadIdx.x == 0) flags[j.inst0 + inst] = 1u;
+        if (__syncthreads_or((int)hit) && threadIdx.x == 0) {
+            flags[j.inst0 + inst] = 1u;
+            *any = 1u;
+        }
     }
 }
 
@@ -384,6 +392,7 @@ __global__ void __launch_bounds__(256) pg_compact(const PgSlot* __restrict__ slo
 __global__ void __launch_bounds__(256) pg_reset_flagged(const u32* flags, u32 n_inst, const u64* inst_slot0,
                                                         u32 kernel, PgSlot* slots, u64* inst_cnt) {
     const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (!flags[n_inst]) return;   // (the batch's any-flagged word)
     if (i >= n_inst || !flags[i]) return;
     inst_cnt[i] = 0ull;
     PgSlot* s = slots + inst_slot0[i] + (u64)kernel * PG_NK;
@@ -419,11 +428,13 @@ namespace pgk {
 static u32 units_grid(u32 max_inst, u32 cap) { return max_inst < cap ? (max_inst ? max_inst : 1u) : cap; }
 
 cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 max_inst, u32* arena_s, u32* arena_t, u32* input,
-                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags) {
+                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags,
+                       const u32* any) {
     for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
         const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
         dim3 grid(units_grid(max_inst, flags ? 8u : 1024u), nj);
-        pg_gen_inputs<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, seed_base, mode, range, mask, flags);
+        pg_gen_inputs<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, seed_base, mode, range, mask, flags,
+                                            any);
     }
     return cudaGetLastError();
 }
@@ -465,11 +476,12 @@ cudaError_t lockstep(const PgLock* jobs, u32 n_jobs, u32 max_inst, const u32* ar
     return cudaGetLastError();
 }
 
-cudaError_t xb_detect(const PgXb* jobs, u32 n_jobs, u32 max_inst, const u32* arena, u32* flags, cudaStream_t st) {
+cudaError_t xb_detect(const PgXb* jobs, u32 n_jobs, u32 max_inst, const u32* arena, u32* flags, u32* any,
+                      cudaStream_t st) {
     for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
         const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
         dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
-        pg_xb_detect<<<grid, 256, 0, st>>>(jobs + j0, arena, flags);
+        pg_xb_detect<<<grid, 256, 0, st>>>(jobs + j0, arena, flags, any);
     }
     return cudaGetLastError();
 }

@@ -103,6 +103,8 @@ struct PgParams {
     const u32* work_count;  // their number (device); nullptr: one item per CTA, or
     u32 n_work;             // (non-zero) a grid-stride loop over this many items (exact re-run)
     u32 pad3;
+    u32* flag_any;          // set when any instance of the batch is flagged; re-run passes with
+                            // nothing flagged exit at once (nullptr: absent)
 };
 
 // K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive
