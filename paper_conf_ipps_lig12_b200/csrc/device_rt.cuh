@@ -623,19 +623,15 @@ __device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, val);
     pg_fcount(t);
 }
-// global arrays: per-seed arenas (values, last writer and the XB block marks are read per
-// instance by K2b/K3); owner and reader stamps agree across the seeds and live in the
-// group's first arena only
+// global arrays: per-seed arenas for values and last writers (read per instance by K2b/K3);
+// owner, reader and XB block stamps agree across the seeds and live in the group's first
+// arena only (K1 initialises them there only, K2b flags the whole group)
 template <int A>
 __device__ __forceinline__ void pg_xb_mark_ms(const PgT& t, u32 flat) {
-    if (pg_sL.nblocks > 1u) {
-        const u64 st = pg_sL.arena_stride;
-        PG_S_LOOP {
-            if (_s < t.nsv) {
-                atomicMin(t.arena + _s * st + PG_ARR(A).off_xf + flat, t.blk + 1u);
-                atomicMax(t.arena + _s * st + PG_ARR(A).off_xl + flat, t.blk + 1u);
-            }
-        }
+    if (pg_sL.nblocks > 1u) {   // (the group's first arena: every seed touches the same cells; K2b
+                                //  decides for the whole group)
+        atomicMin(t.arena + PG_ARR(A).off_xf + flat, t.blk + 1u);
+        atomicMax(t.arena + PG_ARR(A).off_xl + flat, t.blk + 1u);
     }
 }
 template <int A, bool RD, bool LOG>
@@ -811,14 +807,10 @@ __device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 }
 template <int A>
 __device__ __forceinline__ void pg_xb_mark_ms(const PgT& t, u32 flat) {
-    if (pg_sL.nblocks > 1u) {
-        const u64 st = pg_sL.arena_stride;
-        PG_S_LOOP {
-            if (_s < t.nsv) {
-                atomicMin(t.arena + _s * st + PG_ARR(A).off_xf + flat, t.blk + 1u);
-                atomicMax(t.arena + _s * st + PG_ARR(A).off_xl + flat, t.blk + 1u);
-            }
-        }
+    if (pg_sL.nblocks > 1u) {   // (the group's first arena: every seed touches the same cells; K2b
+                                //  decides for the whole group)
+        atomicMin(t.arena + PG_ARR(A).off_xf + flat, t.blk + 1u);
+        atomicMax(t.arena + PG_ARR(A).off_xl + flat, t.blk + 1u);
     }
 }
 template <int A, bool RD, bool LOG>

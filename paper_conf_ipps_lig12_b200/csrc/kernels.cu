@@ -11,61 +11,79 @@
 
 namespace {
 
-__device__ __forceinline__ u32 init_value(u32 mode, u32 range, u32 mask, u64 seed, u32 gid, u32 i) {
+
+
+// CTA tasks of the per-(job, instance) kernels (K1, K2b, K3): jobs carry task0, the index
+// of their first task; a task is a PG_FILL_CHUNK-word chunk of one instance (arrays of more
+// than PG_FILL_SMALL words) or 8 instances, a warp each.  Returns the job of `task`.
+template <class J>
+__device__ __forceinline__ u32 pg_task_job(const J* jobs, u32 n_jobs, u32 task_base, u32 task, u32* s_job) {
+    if (threadIdx.x == 0) {
+        u32 lo = 0, hi = n_jobs - 1u;
+        while (lo < hi) {
+            const u32 mid = (lo + hi + 1u) >> 1;
+            if (jobs[mid].task0 - task_base <= task) lo = mid;
+            else hi = mid - 1u;
+        }
+        *s_job = lo;
+    }
+    __syncthreads();
+    const u32 j = *s_job;
+    __syncthreads();   // (*s_job is rewritten for the next task)
+    return j;
+}
+
+// One CTA task per grid-stride step (tasks of all jobs numbered consecutively, task0 per
+// job): a 4096-word chunk of one instance stored as 128-bit words, or 8 small instances, a
+// warp each.  With `flags`, only flagged instances are (re-)initialised: the exact re-run of
+// the instances the optimistic pass flagged.
+__device__ __forceinline__ u32 fill_value(u32 op, u32 mode, u32 range, u32 mask, u32 value, u64 key, u64 seed,
+                                          u32 i) {
+    if (op == PGF_CONST) return value;
     u32 v;
     if (mode == 1) v = i < 64 ? (u32)((seed >> i) & 1ull) : 0u;                 // BITS01
-    else if (mode == 2) v = pg_rand32(seed, gid, i) % (range ? range : 1u);      // RANGE(k)
-    else v = pg_rand32(seed, gid, i);                                           // RAND32
+    else if (mode == 2) v = pg_rand32_k(key, i) % (range ? range : 1u);          // RANGE(k)
+    else v = pg_rand32_k(key, i);                                               // RAND32
     return v & mask;
 }
-
-// K1: blockIdx.y = job, blockIdx.x strides over the job's instances, threads
-// stride over the words.
-// With `flags`, only the jobs of region `only_target` and only flagged instances are
-// (re-)initialised: the exact re-run of the instances the optimistic pass flagged.
-// Work units of the per-(job, instance) kernels K1/K2b/K3: a CTA per instance for arrays
-// of more than kSmallN words, else a warp per instance (most C1-C4 output arrays hold a
-// few words: a CTA of idle threads per instance would cost more than the words).
-constexpr u32 kSmallN = 512u;
-// Large arrays are cut into chunks of kChunk words, one CTA per (instance, chunk), so one
-// instance's words are spread over many SMs.
-constexpr u32 kChunk = 65536u;
-struct Units {
-    u32 first, step, tid, nthr;   // unit loop (first, step) and word loop (tid, nthr)
-    u32 nchunk;                   // units per instance
-};
-__device__ __forceinline__ Units pg_units(u32 n) {
-    if (n > kSmallN) return Units{blockIdx.x, gridDim.x, threadIdx.x, blockDim.x, (n + kChunk - 1u) / kChunk};
-    const u32 nw = blockDim.x >> 5;
-    return Units{blockIdx.x * nw + (threadIdx.x >> 5), gridDim.x * nw, threadIdx.x & 31u, 32u, 1u};
-}
-// words [w0, w1) of unit `un` (instance un / nchunk)
-__device__ __forceinline__ void pg_unit_words(const Units& u, u32 un, u32 n, u32& inst, u32& w0, u32& w1) {
-    inst = un / u.nchunk;
-    w0 = (un - inst * u.nchunk) * kChunk;
-    w1 = u.nchunk == 1u ? n : min(n, w0 + kChunk);
-    if (u.nchunk == 1u) w0 = 0u;
-}
-
-// (with `flags`, only flagged instances are (re-)initialised: the exact re-run of the
-// instances the optimistic pass flagged)
-__global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ jobs, u32* arena_s, u32* arena_t,
-                                                     u32* input, u64 seed_base, u32 mode, u32 range, u32 mask,
+__global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ jobs, u32 n_jobs, u32 task_base,
+                                                     u32 n_tasks, u32* arena_s, u32* arena_t, u32* input,
+                                                     u64 seed_base, u32 mode, u32 range, u32 mask,
                                                      const u32* flags, const u32* any) {
     if (flags && !*any) return;   // re-initialisation with nothing flagged
-    const PgFill f = jobs[blockIdx.y];
-    u32* region = f.target == 0 ? arena_s : f.target == 1 ? arena_t : input;
-    const Units u = pg_units(f.n);
-    for (u32 un = u.first; un < f.n_inst * u.nchunk; un += u.step) {
-        u32 inst, w0, w1;
-        pg_unit_words(u, un, f.n, inst, w0, w1);
-        if (flags && !flags[f.inst0 + inst]) continue;
-        u32* base = region + f.dst + (u64)inst * f.stride;
-        const u64 seed = seed_base + (u64)f.j0 + (u64)inst * f.jstep;
-        if (f.op == PGF_CONST) {
-            for (u32 i = w0 + u.tid; i < w1; i += u.nthr) base[i] = f.value;
-        } else {  // PGF_INPUT (initial values of an input region or of a written array)
-            for (u32 i = w0 + u.tid; i < w1; i += u.nthr) base[i] = init_value(mode, range, mask, seed, f.gid, i);
+    __shared__ u32 s_job;
+    for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
+        const PgFill f = jobs[pg_task_job(jobs, n_jobs, task_base, task, &s_job)];
+        const u32 lt = task - (f.task0 - task_base);
+        u32* region = f.target == 0 ? arena_s : f.target == 1 ? arena_t : input;
+        if (f.n > PG_FILL_SMALL) {
+            const u32 nch = (f.n + PG_FILL_CHUNK - 1u) / PG_FILL_CHUNK;
+            const u32 inst = lt / nch, w0 = (lt - inst * nch) * PG_FILL_CHUNK;
+            const u32 w1 = min(f.n, w0 + PG_FILL_CHUNK);
+            const u32 ai = inst * f.istep;
+            if (flags && !flags[f.inst0 + ai]) continue;
+            u32* base = region + f.dst + (u64)ai * f.stride;   // (128-byte aligned: arena layout)
+            const u64 seed = seed_base + (u64)f.j0 + (u64)ai * f.jstep;
+            const u64 key = pg_sm64(seed) ^ ((u64)f.gid << 48);
+            const u32 w4 = w0 + ((w1 - w0) & ~3u);
+            for (u32 i = w0 + 4u * threadIdx.x; i < w4; i += 4u * blockDim.x) {
+                uint4 q;
+                q.x = fill_value(f.op, mode, range, mask, f.value, key, seed, i);
+                q.y = fill_value(f.op, mode, range, mask, f.value, key, seed, i + 1u);
+                q.z = fill_value(f.op, mode, range, mask, f.value, key, seed, i + 2u);
+                q.w = fill_value(f.op, mode, range, mask, f.value, key, seed, i + 3u);
+                *(uint4*)(base + i) = q;
+            }
+            for (u32 i = w4 + threadIdx.x; i < w1; i += blockDim.x)
+                base[i] = fill_value(f.op, mode, range, mask, f.value, key, seed, i);
+        } else {
+            const u32 inst = lt * 8u + (threadIdx.x >> 5), lane = threadIdx.x & 31u;
+            const u32 ai = inst * f.istep;
+            if (inst >= f.n_inst || (flags && !flags[f.inst0 + ai])) continue;
+            u32* base = region + f.dst + (u64)ai * f.stride;
+            const u64 seed = seed_base + (u64)f.j0 + (u64)ai * f.jstep;
+            const u64 key = pg_sm64(seed) ^ ((u64)f.gid << 48);
+            for (u32 i = lane; i < f.n; i += 32u) base[i] = fill_value(f.op, mode, range, mask, f.value, key, seed, i);
         }
     }
 }
@@ -73,36 +91,36 @@ __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ 
 __device__ __forceinline__ u32 cmp_val(const u32* region, u32 kind, u64 off, u32 i) { return region[off + i]; }
 
 // K3a: count mismatching cells per (instance, array); keep the minimum (gid, addr)
-// per instance.
-__global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs, const u32* arena_s,
-                                                  const u32* arena_t, const u32* input, PgSlot* slots,
-                                                  u64* mm_key) {
+// per instance.  One CTA task per grid-stride step (pg_task_job).
+__global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs, u32 n_jobs, u32 n_tasks,
+                                                  const u32* arena_s, const u32* arena_t, const u32* input,
+                                                  PgSlot* slots, u64* mm_key) {
     __shared__ u32 s_cnt;
     __shared__ u32 s_min;
-    const PgCmp c = jobs[blockIdx.y];
-    const u32* rs = c.src_kind == 0 ? arena_s : input;
-    const u32* rt = c.tgt_kind == 0 ? arena_t : input;
-    if (c.n <= kSmallN) {   // a warp per instance
-        const Units u = pg_units(c.n);
-        for (u32 inst = u.first; inst < c.n_inst; inst += u.step) {
+    __shared__ u32 s_job;
+    for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
+        const PgCmp c = jobs[pg_task_job(jobs, n_jobs, 0u, task, &s_job)];
+        const u32 lt = task - c.task0;
+        const u32* rs = c.src_kind == 0 ? arena_s : input;
+        const u32* rt = c.tgt_kind == 0 ? arena_t : input;
+        if (c.n <= PG_FILL_SMALL) {   // a warp per instance
+            const u32 inst = lt * 8u + (threadIdx.x >> 5), lane = threadIdx.x & 31u;
+            if (inst >= c.n_inst) continue;
             const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
             u32 cnt = 0, mn = PG_NEVER;
-            for (u32 i = u.tid; i < c.n; i += 32u) {
+            for (u32 i = lane; i < c.n; i += 32u) {
                 if (cmp_val(rs, c.src_kind, so, i) != cmp_val(rt, c.tgt_kind, to, i)) { cnt++; mn = min(mn, i); }
             }
             cnt = __reduce_add_sync(0xffffffffu, cnt);
             mn = __reduce_min_sync(0xffffffffu, mn);
-            if (u.tid == 0 && cnt) {
+            if (lane == 0 && cnt) {
                 atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step].count, (u64)cnt);
                 atomicMin(&mm_key[c.inst0 + inst], ((u64)c.gid << 32) | mn);
             }
+            continue;
         }
-        return;
-    }
-    const Units u = pg_units(c.n);
-    for (u32 un = u.first; un < c.n_inst * u.nchunk; un += u.step) {
-        u32 inst, w0, w1;
-        pg_unit_words(u, un, c.n, inst, w0, w1);
+        const u32 nch = (c.n + PG_FILL_CHUNK - 1u) / PG_FILL_CHUNK;
+        const u32 inst = lt / nch, w0 = (lt - inst * nch) * PG_FILL_CHUNK, w1 = min(c.n, w0 + PG_FILL_CHUNK);
         if (threadIdx.x == 0) { s_cnt = 0; s_min = PG_NEVER; }
         __syncthreads();
         const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
@@ -149,39 +167,39 @@ __global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__
 
 // K2b: flag every instance in which some global cell written by the kernel was
 // accessed by two blocks (X4 XB) - the block-parallel pass is not exact there.
-__global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ jobs, const u32* arena, u32* flags,
-                                                    u32* any) {
-    const PgXb j = jobs[blockIdx.y];
-    if (j.n <= kSmallN) {   // a warp per instance
-        const Units u = pg_units(j.n);
-        for (u32 inst = u.first; inst < j.n_inst; inst += u.step) {
-            const u64 base = (u64)inst * j.stride;
+__global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ jobs, u32 n_jobs, u32 n_tasks,
+                                                    const u32* arena, u32* flags, u32* any) {
+    __shared__ u32 s_job;
+    for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
+        const PgXb j = jobs[pg_task_job(jobs, n_jobs, 0u, task, &s_job)];
+        const u32 lt = task - j.task0;
+        const u32 nb = (j.n_inst + j.istep - 1u) / j.istep;   // instances holding marks
+        auto flag = [&](u32 b) {   // the group of instance b * istep
+            const u32 i0 = b * j.istep, i1 = min(j.n_inst, i0 + j.istep);
+            for (u32 i = i0; i < i1; i++) flags[j.inst0 + i] = 1u;
+            *any = 1u;
+        };
+        if (j.n <= PG_FILL_SMALL) {   // a warp per instance
+            const u32 b = lt * 8u + (threadIdx.x >> 5), lane = threadIdx.x & 31u;
+            if (b >= nb) continue;
+            const u64 base = (u64)b * j.istep * j.stride;
             u32 hit = 0;
-            for (u32 i = u.tid; i < j.n; i += 32u) {
+            for (u32 i = lane; i < j.n; i += 32u) {
                 const u32 xf = arena[j.xf + base + i], xl = arena[j.xl + base + i];
                 hit |= (xl != 0u && xf != xl && arena[j.lw + base + i] != 0u);
             }
-            if (__any_sync(0xffffffffu, hit) && u.tid == 0) {
-                flags[j.inst0 + inst] = 1u;
-                *any = 1u;
-            }
+            if (__any_sync(0xffffffffu, hit) && lane == 0) flag(b);
+            continue;
         }
-        return;
-    }
-    const Units u = pg_units(j.n);
-    for (u32 un = u.first; un < j.n_inst * u.nchunk; un += u.step) {
-        u32 inst, w0, w1;
-        pg_unit_words(u, un, j.n, inst, w0, w1);
-        const u64 base = (u64)inst * j.stride;
+        const u32 nch = (j.n + PG_FILL_CHUNK - 1u) / PG_FILL_CHUNK;
+        const u32 b = lt / nch, w0 = (lt - b * nch) * PG_FILL_CHUNK, w1 = min(j.n, w0 + PG_FILL_CHUNK);
+        const u64 base = (u64)b * j.istep * j.stride;
         u32 hit = 0;
         for (u32 i = w0 + threadIdx.x; i < w1; i += blockDim.x) {
             const u32 xf = arena[j.xf + base + i], xl = arena[j.xl + base + i], lw = arena[j.lw + base + i];
             hit |= (xl != 0u) & (xf != xl) & (lw != 0u);
         }
-        if (__syncthreads_or((int)hit) && threadIdx.x == 0) {
-            flags[j.inst0 + inst] = 1u;
-            *any = 1u;
-        }
+        if (__syncthreads_or((int)hit) && threadIdx.x == 0) flag(b);
     }
 }
 
@@ -425,17 +443,15 @@ namespace pgk {
 
 // grid.x of the per-(job, instance) kernels: enough CTAs for a CTA per instance, capped
 // (re-initialisation of flagged instances: a few CTAs per job walk its instances)
-static u32 units_grid(u32 max_inst, u32 cap) { return max_inst < cap ? (max_inst ? max_inst : 1u) : cap; }
 
-cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 max_inst, u32* arena_s, u32* arena_t, u32* input,
-                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags,
+
+cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 task_base, u32 n_tasks, u32* arena_s, u32* arena_t,
+                       u32* input, u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags,
                        const u32* any) {
-    for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
-        const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
-        dim3 grid(units_grid(max_inst, flags ? 8u : 1024u), nj);
-        pg_gen_inputs<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, seed_base, mode, range, mask, flags,
-                                            any);
-    }
+    if (!n_jobs || !n_tasks) return cudaSuccess;
+    const u32 grid = n_tasks < 148u * 16u ? n_tasks : 148u * 16u;
+    pg_gen_inputs<<<grid, 256, 0, st>>>(jobs, n_jobs, task_base, n_tasks, arena_s, arena_t, input, seed_base, mode,
+                                        range, mask, flags, any);
     return cudaGetLastError();
 }
 
@@ -452,12 +468,13 @@ cudaError_t count_reduce(const u64* inst_cnt, u32 n, long long* counts, cudaStre
     return cudaGetLastError();
 }
 
-cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 max_inst, const u32* arena_s, const u32* arena_t,
-                    const u32* input, PgSlot* slots, u64* mm_key, cudaStream_t st) {
+cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 n_tasks, u32 max_inst, const u32* arena_s,
+                    const u32* arena_t, const u32* input, PgSlot* slots, u64* mm_key, cudaStream_t st) {
+    if (!n_jobs) return cudaSuccess;
+    pg_compare<<<n_tasks < 148u * 16u ? n_tasks : 148u * 16u, 256, 0, st>>>(jobs, n_jobs, n_tasks, arena_s, arena_t,
+                                                                            input, slots, mm_key);
     for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
         const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
-        dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
-        pg_compare<<<grid, 256, 0, st>>>(jobs + j0, arena_s, arena_t, input, slots, mm_key);
         dim3 g2((max_inst + 127) / 128, nj);
         pg_compare_fill<<<g2, 128, 0, st>>>(jobs + j0, arena_s, arena_t, input, slots, mm_key);
     }
@@ -476,13 +493,11 @@ cudaError_t lockstep(const PgLock* jobs, u32 n_jobs, u32 max_inst, const u32* ar
     return cudaGetLastError();
 }
 
-cudaError_t xb_detect(const PgXb* jobs, u32 n_jobs, u32 max_inst, const u32* arena, u32* flags, u32* any,
+cudaError_t xb_detect(const PgXb* jobs, u32 n_jobs, u32 n_tasks, const u32* arena, u32* flags, u32* any,
                       cudaStream_t st) {
-    for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
-        const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
-        dim3 grid(max_inst < 1024u ? max_inst : 1024u, nj);
-        pg_xb_detect<<<grid, 256, 0, st>>>(jobs + j0, arena, flags, any);
-    }
+    if (!n_jobs || !n_tasks) return cudaSuccess;
+    pg_xb_detect<<<n_tasks < 148u * 16u ? n_tasks : 148u * 16u, 256, 0, st>>>(jobs, n_jobs, n_tasks, arena, flags,
+                                                                              any);
     return cudaGetLastError();
 }
 

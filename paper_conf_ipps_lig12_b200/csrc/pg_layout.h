@@ -121,8 +121,20 @@ struct PgFill {
     u32 value;    // PGF_CONST fill value
     u32 target;   // 0 arena (src), 1 arena (tgt), 2 input region
     u32 inst0;    // batch-local index of instance 0 (re-initialisation of flagged instances)
+    u32 task0;    // first CTA task of this job in the batch's fill list (pg_fill_tasks)
+    u32 istep;    // instances 0, istep, 2 istep, ... (n_inst of them): stamps that only the first
+                  // instance of a multi-seed group keeps
     u32 pad;
 };
+// CTA tasks of a K1 job: a chunk of PG_FILL_CHUNK words of one instance (arrays of more than
+// PG_FILL_SMALL words), else 8 instances (a warp each)
+#define PG_FILL_CHUNK 4096u
+#define PG_FILL_SMALL 512u
+#ifndef __CUDACC_RTC__
+static inline u32 pg_fill_tasks(u32 n, u32 n_inst) {
+    return n > PG_FILL_SMALL ? n_inst * ((n + PG_FILL_CHUNK - 1u) / PG_FILL_CHUNK) : (n_inst + 7u) / 8u;
+}
+#endif
 
 // K2b (pg_xb_detect) job: one global array written by a kernel, for n_inst
 // consecutive instances of one launch: flags instances whose cells were
@@ -130,7 +142,10 @@ struct PgFill {
 struct PgXb {
     u64 xf, xl, lw;   // u32-word offsets of instance 0 in the kernel arena
     u64 stride;
-    u32 n, n_inst, inst0, pad;
+    u32 n, n_inst, inst0;
+    u32 istep;        // multi-seed launches: the marks live in the first instance of each group of
+                      // istep seeds, whose verdict holds for the whole group
+    u32 task0, pad;   // first CTA task (pg_fill_tasks over the instances holding marks)
 };
 
 // K3b (pg_lockstep) job: one shared array both kernels of a pair declare (same name
@@ -150,4 +165,5 @@ struct PgCmp {
     u64 src_lw, tgt_lw;          // last-writer words of instance 0 (kind 0 only)
     u64 slot0, slot_step;        // MISMATCH slot of (instance 0, kernel 0) and stride
     u32 inst0, n_inst, gid, n, src_kind, tgt_kind;
+    u32 task0, pad;              // first CTA task (pg_fill_tasks(n, n_inst))
 };

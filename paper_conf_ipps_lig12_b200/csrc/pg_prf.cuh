@@ -12,3 +12,7 @@ __device__ __forceinline__ unsigned int pg_rand32(unsigned long long seed, unsig
                                                   unsigned long long idx) {
     return (unsigned int)pg_sm64(pg_sm64(seed) ^ (tag << 48) ^ idx);
 }
+// the same with sm(seed) ^ (tag << 48) computed once per (seed, array)
+__device__ __forceinline__ unsigned int pg_rand32_k(unsigned long long key, unsigned long long idx) {
+    return (unsigned int)pg_sm64(key ^ idx);
+}
