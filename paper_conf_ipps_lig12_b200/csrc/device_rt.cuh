@@ -1372,6 +1372,124 @@ __device__ __noinline__ void pg_flush_cta(const PgParams& P, u32 lane, u32 warp,
     }
 }
 
+#if PG_MSX
+// Record flush of the multi-seed exact pass: every event of this pass carries the recording
+// thread's gtid as tid_a (OOB, UNINIT, LIMIT, WW and RW alike), so two candidates never tie
+// on the seed-independent fields (round, array, addr, tid_a, tid_b, site); the merge runs
+// once per kind on those fields and the winner's per-seed values fill the seeds' slots.  The
+// group's first slot's lock guards all of its seeds' slots (always updated together).
+struct PgFlushEntryMs {
+    u64 slot;       // ~0: empty
+    u32 cnt, nsv;
+    u32 f[6];
+    u32 v[PG_MS][2];
+};
+__device__ __noinline__ void pg_slot_update_ms(PgSlot* s0, u64 step, u32 nsv, u32 cnt, const u32* f6,
+                                               const u32 (*v)[2]) {
+    for (u32 q = 0; q < nsv; q++) atomicAdd(&s0[q * step].count, (u64)cnt);
+    while (atomicCAS(&s0->lock, 0u, 1u) != 0u) {
+    }
+    __threadfence();
+    volatile PgSlot* vs = s0;
+    bool less = !vs->has;
+    if (!less) {
+        for (int i = 0; i < 6; i++) {
+            const u32 cur = vs->f[i];
+            if (f6[i] != cur) {
+                less = f6[i] < cur;
+                break;
+            }
+        }
+    }
+    if (less) {
+        for (u32 q = 0; q < nsv; q++) {
+            volatile PgSlot* t = s0 + q * step;
+#pragma unroll
+            for (int i = 0; i < 6; i++) t->f[i] = f6[i];
+            t->f[6] = v[q][0];
+            t->f[7] = v[q][1];
+            t->has = 1u;
+        }
+    }
+    __threadfence();
+    atomicExch(&s0->lock, 0u);
+}
+__device__ __noinline__ void pg_flush_cta_ms(const PgParams& P, u32 lane, u32 warp, PgCold& c, u32 evm, u32 valid,
+                                             u64 slot0, u32 nsv, PgFlushEntryMs* sh /* [32] */, u32 kmask) {
+    const u32 nwarps = blockDim.x >> 5;
+    const u64 step = pg_sW.slot_step;
+    for (u32 k = 0; k < PG_NK; k++) {
+        if (!((kmask >> k) & 1u)) continue;
+        if (lane == 0) sh[warp].slot = ~0ull;
+        __syncwarp();
+        u32 pending = valid && ((evm >> k) & 1u);
+        bool first = true;
+        for (;;) {
+            if (!__any_sync(PG_FULL, pending)) break;
+            u32 leader, cnt, members, best[8];
+            u64 key;
+            u32 f_in[8];
+#pragma unroll
+            for (int i = 0; i < 6; i++) f_in[i] = pending ? c.ebest[k][i] : PG_NEVER;
+            f_in[6] = f_in[7] = pending ? 0u : PG_NEVER;
+            pg_warp_merge(pending, slot0, pending ? c.ecnt[k] : 0u, f_in, lane, leader, key, cnt, best, members);
+            bool same = pending && slot0 == key;
+#pragma unroll
+            for (int i = 0; i < 6; i++) same = same && f_in[i] == best[i];
+            const u32 win = (u32)__ffs(__ballot_sync(PG_FULL, same)) - 1u;
+            u32 vv[PG_MS][2];
+#pragma unroll
+            for (u32 q = 0; q < PG_MS; q++) {
+                vv[q][0] = __shfl_sync(PG_FULL, c.ebv[k][q][0], win);
+                vv[q][1] = __shfl_sync(PG_FULL, c.ebv[k][q][1], win);
+            }
+            const u32 wn = __shfl_sync(PG_FULL, nsv, win);
+            if (lane == leader) {
+                if (first) {   // the common case: one group per warp -> deposit for the CTA merge
+                    sh[warp].slot = key;
+                    sh[warp].cnt = cnt;
+                    sh[warp].nsv = wn;
+#pragma unroll
+                    for (int i = 0; i < 6; i++) sh[warp].f[i] = best[i];
+#pragma unroll
+                    for (u32 q = 0; q < PG_MS; q++) { sh[warp].v[q][0] = vv[q][0]; sh[warp].v[q][1] = vv[q][1]; }
+                } else {
+                    pg_slot_update_ms(P.slots + key + k, step, wn, cnt, best, vv);
+                }
+            }
+            first = false;
+            if (members & (1u << lane)) pending = 0u;
+            __syncwarp();
+        }
+        __syncthreads();
+        if (warp == 0) {
+            const bool has = lane < nwarps && sh[lane].slot != ~0ull;
+            u32 pend = has;
+            const u64 skey = has ? sh[lane].slot : 0ull;
+            const u32 scnt = has ? sh[lane].cnt : 0u;
+            u32 sf[8];
+#pragma unroll
+            for (int i = 0; i < 6; i++) sf[i] = has ? sh[lane].f[i] : PG_NEVER;
+            sf[6] = sf[7] = has ? 0u : PG_NEVER;
+            for (;;) {
+                if (!__any_sync(PG_FULL, pend)) break;
+                u32 leader, cnt, members, best[8];
+                u64 key;
+                pg_warp_merge(pend, skey, scnt, sf, lane, leader, key, cnt, best, members);
+                bool same = pend && skey == key;
+#pragma unroll
+                for (int i = 0; i < 6; i++) same = same && sf[i] == best[i];
+                const u32 win = (u32)__ffs(__ballot_sync(PG_FULL, same)) - 1u;
+                if (lane == leader) pg_slot_update_ms(P.slots + key + k, step, sh[win].nsv, cnt, best, sh[win].v);
+                if (members & (1u << lane)) pend = 0u;
+                __syncwarp();
+            }
+        }
+        __syncthreads();
+    }
+}
+#endif
+
 // ------------------------------------------------------------------ CTA main loop
 // A CTA runs G groups of one launch in lock step.  Group g emulates, for seed
 // (g / gb) of the work item, the blocks blk0 + i*gb + (g % gb), i = 0, 1, ...
@@ -1717,9 +1835,9 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
 #if PG_MSX
-                for (u32 q = 0; q < PG_MS; q++)   // one slot per seed of the group
-                    pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_ && q < nsv,
-                                 pg_sW.slot0 + (u64)(sb + q) * pg_sW.slot_step, s_flush, kmask, q);
+                __shared__ PgFlushEntryMs s_flush_ms[32];
+                pg_flush_cta_ms(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_,
+                                pg_sW.slot0 + (u64)sb * pg_sW.slot_step, nsv, s_flush_ms, kmask);
 #else
                 pg_flush_cta(P, lane, warp, Cd[v], T[v].evm, inst_ok && T[v].tlin < T_, pg_sW.slot0 + (u64)sb * pg_sW.slot_step,
                              s_flush, kmask);

@@ -19,7 +19,16 @@ namespace {
 template <class J>
 __device__ __forceinline__ u32 pg_task_job(const J* jobs, u32 n_jobs, u32 task_base, u32 task, u32* s_job) {
     if (threadIdx.x == 0) {
-        u32 lo = 0, hi = n_jobs - 1u;
+        // a CTA visits its tasks in increasing order, so the job index never decreases:
+        // gallop forward from the last job found, then bisect
+        u32 lo = *s_job < n_jobs ? *s_job : 0u, hi = lo, d = 1;
+        while (hi + 1u < n_jobs && jobs[hi + 1u].task0 - task_base <= task) {
+            lo = hi + 1u;
+            hi = min(n_jobs - 1u, hi + d);
+            d <<= 1;
+            if (jobs[hi].task0 - task_base > task) { hi -= 1u; break; }
+            lo = hi;
+        }
         while (lo < hi) {
             const u32 mid = (lo + hi + 1u) >> 1;
             if (jobs[mid].task0 - task_base <= task) lo = mid;
@@ -29,7 +38,7 @@ __device__ __forceinline__ u32 pg_task_job(const J* jobs, u32 n_jobs, u32 task_b
     }
     __syncthreads();
     const u32 j = *s_job;
-    __syncthreads();   // (*s_job is rewritten for the next task)
+    __syncthreads();   // (thread 0 rewrites *s_job for the next task)
     return j;
 }
 
@@ -52,6 +61,7 @@ __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ 
                                                      const u32* flags, const u32* any) {
     if (flags && !*any) return;   // re-initialisation with nothing flagged
     __shared__ u32 s_job;
+    if (threadIdx.x == 0) s_job = 0u;
     for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
         const PgFill f = jobs[pg_task_job(jobs, n_jobs, task_base, task, &s_job)];
         const u32 lt = task - (f.task0 - task_base);
@@ -98,6 +108,7 @@ __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs
     __shared__ u32 s_cnt;
     __shared__ u32 s_min;
     __shared__ u32 s_job;
+    if (threadIdx.x == 0) s_job = 0u;
     for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
         const PgCmp c = jobs[pg_task_job(jobs, n_jobs, 0u, task, &s_job)];
         const u32 lt = task - c.task0;
@@ -170,6 +181,7 @@ __global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__
 __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ jobs, u32 n_jobs, u32 n_tasks,
                                                     const u32* arena, u32* flags, u32* any) {
     __shared__ u32 s_job;
+    if (threadIdx.x == 0) s_job = 0u;
     for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
         const PgXb j = jobs[pg_task_job(jobs, n_jobs, 0u, task, &s_job)];
         const u32 lt = task - j.task0;

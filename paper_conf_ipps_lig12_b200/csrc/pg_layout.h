@@ -128,7 +128,7 @@ struct PgFill {
 };
 // CTA tasks of a K1 job: a chunk of PG_FILL_CHUNK words of one instance (arrays of more than
 // PG_FILL_SMALL words), else 8 instances (a warp each)
-#define PG_FILL_CHUNK 4096u
+#define PG_FILL_CHUNK 16384u
 #define PG_FILL_SMALL 512u
 #ifndef __CUDACC_RTC__
 static inline u32 pg_fill_tasks(u32 n, u32 n_inst) {
