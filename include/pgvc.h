@@ -173,6 +173,13 @@ int pg_collect_lockstep(pg_run *r, uint32_t *rows, size_t cap_rows, size_t *n_ro
 
 /* Introspection of a loaded kernel. */
 int pg_ir_info(const pg_ir *k, uint32_t *n_sites, uint32_t *n_globals, uint32_t *n_scalars);
+/* *oblivious = 1 when no address, access guard, branch or loop condition of the kernel
+ * depends on array contents (no private arrays either): every seed of a launch then takes
+ * the same accesses in the same rounds, and the optimistic and exact passes run several
+ * seeds per lane (multi-seed lanes); 0 otherwise (e.g. the bitonic
+ * compare-exchange, whose store guard depends on the data).  *n_tainted = the variables
+ * that may hold an input-dependent value.  PG_E_ARG on a null kernel. */
+int pg_ir_seed_oblivious(const pg_ir *k, uint32_t *oblivious, uint32_t *n_tainted);
 /* Generated CUDA source of the evaluation kernel for (bits, checks, bank_model). */
 int pg_ir_source(const pg_ir *k, uint32_t bits, uint32_t checks, uint32_t bank_model, char *buf, size_t cap,
                  size_t *len);

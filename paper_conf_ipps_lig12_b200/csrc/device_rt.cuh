@@ -559,7 +559,13 @@ __device__ __forceinline__ void pg_st_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32
 // would be an event (OOB, UNINIT, LIMIT, a race) flags the group's instances, which the
 // exact single-seed re-run then evaluates and records.
 __device__ __forceinline__ void pg_vld(const u32* p, u32 (&v)[PG_MS]) {
-#if PG_MS == 8
+#if PG_MS == 16
+#pragma unroll
+    for (int h = 0; h < 4; h++) {
+        const uint4 q = *(const uint4*)(p + 4 * h);
+        v[4 * h] = q.x; v[4 * h + 1] = q.y; v[4 * h + 2] = q.z; v[4 * h + 3] = q.w;
+    }
+#elif PG_MS == 8
     const uint4 q = *(const uint4*)p, r = *(const uint4*)(p + 4);
     v[0] = q.x; v[1] = q.y; v[2] = q.z; v[3] = q.w; v[4] = r.x; v[5] = r.y; v[6] = r.z; v[7] = r.w;
 #elif PG_MS == 4
@@ -573,7 +579,10 @@ __device__ __forceinline__ void pg_vld(const u32* p, u32 (&v)[PG_MS]) {
 #endif
 }
 __device__ __forceinline__ void pg_vst(u32* p, const u32 (&v)[PG_MS]) {
-#if PG_MS == 8
+#if PG_MS == 16
+#pragma unroll
+    for (int h = 0; h < 4; h++) *(uint4*)(p + 4 * h) = make_uint4(v[4 * h], v[4 * h + 1], v[4 * h + 2], v[4 * h + 3]);
+#elif PG_MS == 8
     *(uint4*)p = make_uint4(v[0], v[1], v[2], v[3]);
     *(uint4*)(p + 4) = make_uint4(v[4], v[5], v[6], v[7]);
 #elif PG_MS == 4

@@ -75,8 +75,8 @@ class PgError(RuntimeError):
 
 _lib = None
 EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
-           "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_source",
-           "pg_ir_compile", "pg_run_timing", "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
+           "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_seed_oblivious",
+           "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
 
 
 def lib():
@@ -103,6 +103,7 @@ def lib():
                                       ctypes.POINTER(ctypes.c_size_t)]
     L.pg_ir_info.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32),
                              ctypes.POINTER(ctypes.c_uint32)]
+    L.pg_ir_seed_oblivious.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32)]
     L.pg_ir_source.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_char_p,
                                ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]
     L.pg_ir_compile.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32]
@@ -113,8 +114,8 @@ def lib():
     L.pg_ir_free.argtypes = [vp]
     L.pg_run_free.argtypes = [vp]
     for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
-              "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_source",
-              "pg_ir_compile", "pg_run_timing"):
+              "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info",
+              "pg_ir_seed_oblivious", "pg_ir_source", "pg_ir_compile", "pg_run_timing"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -142,6 +143,12 @@ class Ir:
         s, g, c = ctypes.c_uint32(), ctypes.c_uint32(), ctypes.c_uint32()
         _ck(lib().pg_ir_info(self._h, ctypes.byref(s), ctypes.byref(g), ctypes.byref(c)))
         return {"sites": s.value, "globals": g.value, "scalars": c.value}
+
+    def seed_oblivious(self):
+        """(oblivious, n_tainted): pg_ir_seed_oblivious."""
+        o, n = ctypes.c_uint32(), ctypes.c_uint32()
+        _ck(lib().pg_ir_seed_oblivious(self._h, ctypes.byref(o), ctypes.byref(n)))
+        return bool(o.value), n.value
 
     def source(self, bits=32, checks=CHK_RACE | CHK_OOB, bank_model=0) -> str:
         n = ctypes.c_size_t()

@@ -87,3 +87,37 @@ def test_no_cpu_fallback(pgvc):
     with pytest.raises(pgvc.PgError) as e:
         pgvc.check_races(ir, pgvc.Space([((1, 1, 1), (2, 2, 1), (2, 2))]))
     assert e.value.code == pgvc.PG_E_CUDA
+
+
+# ---------------------------------------------------------------- seed-oblivious analysis (multi-seed lanes)
+def test_seed_oblivious_subjects(pgvc, W):
+    """Every reduction, scan, transpose, matmul and post-condition kernel takes the same
+    accesses for every input; the bitonic networks do not (the compare-exchange stores are
+    guarded by the data)."""
+    subj = sorted(f[:-4] for f in os.listdir(os.path.join(ROOT, "subjects")) if f.endswith(".pgk"))
+    for name in subj:
+        ob, nt = pgvc.load_ir(W.subject(name)).seed_oblivious()
+        assert ob == (not name.startswith("bitonic")), name
+    # reduce3 carries mySum (input-dependent); reduce1 keeps only loop counters and indices
+    assert pgvc.load_ir(W.subject("reduce3")).seed_oblivious()[1] >= 1
+    assert pgvc.load_ir(W.subject("reduce1")).seed_oblivious()[1] == 0
+
+
+@pytest.mark.parametrize("body,oblivious", [
+    # data only flows into values: oblivious
+    ("b[t] = a[t] > 0 ? 1 : 2;", True),
+    ("int x = a[t]; int y = x * 3 + t; b[t] = y % 7;", True),
+    # an input-dependent address
+    ("b[a[t] % n] = 1;", False),
+    ("int x = a[t]; b[t] = a[x & 3];", False),
+    # an input-dependent guard of a store, of a load, a loop bound
+    ("if (a[t] > 0) b[t] = 1;", False),
+    ("b[t] = a[t] > 0 ? a[0] : 2;", False),
+    ("int k = a[t] & 7; for (int i = 0; i < k; i++) b[t] = i;", False),
+    # taint through a variable assigned in a loop
+    ("int s = 0; for (int i = 0; i < 4; i++) s = s + a[i]; if (s > 0) b[t] = 1;", False),
+])
+def test_seed_oblivious_cases(pgvc, body, oblivious):
+    text = ("kernel k(global in int a[n], global out int b[n], unsigned n) {\n"
+            "  unsigned t = tid.x;\n  %s\n}\n" % body)
+    assert pgvc.load_ir(text).seed_oblivious()[0] == oblivious
