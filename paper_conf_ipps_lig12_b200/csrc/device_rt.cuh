@@ -245,21 +245,27 @@ __shared__ u32 pg_sAbort;   // some thread of the CTA flagged (CTA-wide blocks)
 #endif
 
 // ------------------------------------------------------------------ bank / coalescing (X9, H6)
-__device__ __forceinline__ void pg_site_stat(u64* st, u32 space, u32 bad, u32 metric, u32 ideal, u32 lanes) {
+// wgt: instances this warp access stands for (multi-seed lanes: the group's seeds)
+__device__ __forceinline__ void pg_site_stat(u64* st, u32 space, u32 bad, u32 metric, u32 ideal, u32 lanes, u32 wgt) {
     // [space, n_acc, n_bad, max, sum, sum_ideal, sum_lanes, 0]
     st[0] = space;
-    atomicAdd(&st[1], 1ull);
-    if (bad) atomicAdd(&st[2], 1ull);
+    atomicAdd(&st[1], (u64)wgt);
+    if (bad) atomicAdd(&st[2], (u64)wgt);
     atomicMax(&st[3], (u64)metric);
-    atomicAdd(&st[4], (u64)metric);
-    atomicAdd(&st[5], (u64)ideal);
-    atomicAdd(&st[6], (u64)lanes);
+    atomicAdd(&st[4], (u64)metric * wgt);
+    atomicAdd(&st[5], (u64)ideal * wgt);
+    atomicAdd(&st[6], (u64)lanes * wgt);
 }
+#if PG_MSX
+#define PG_EVENT_RAW(c, evm, ...) pg_event_msc((c), (evm), __VA_ARGS__)
+#else
+#define PG_EVENT_RAW(c, evm, ...) pg_event((c), (evm), __VA_ARGS__)
+#endif
 
 // All 32 lanes of the warp call these together (the generated code keeps warps
 // converged around every access site).
 __device__ __noinline__ u32 pg_bank_shared(u32 round, u32 lane, u32 ekey0, u32 tlin, u32 gtid, PgCold& c, u32 evm,
-                                           u64* sstats, u32 active, u32 rec, u32 flat, u32 site) {
+                                           u64* sstats, u32 active, u32 rec, u32 flat, u32 site, u32 wgt = 1u) {
     u32 ekey = ekey0;
     if (PG_BANK16) ekey = ekey * 2u + ((tlin >> 4) & 1u);
     const u32 seg = __match_any_sync(PG_FULL, ekey);
@@ -277,14 +283,14 @@ __device__ __noinline__ u32 pg_bank_shared(u32 round, u32 lane, u32 ekey0, u32 t
     const u32 ta = __reduce_min_sync(seg, (active && flat == astar) ? gtid : PG_NEVER);
     const u32 tb = __reduce_min_sync(seg, (active && bank == bstar && flat != astar) ? gtid : PG_NEVER);
     if (amask && lane == (u32)(__ffs(amask) - 1)) {
-        if (sstats && site < PG_NSTATS) pg_site_stat(sstats + site * 8, 1, deg > 1, deg, 1, __popc(amask));
-        if (deg > 1) return pg_event(c, evm, PGK_BANK, round, rec, astar, ta, tb, site, deg, 0);
+        if (sstats && site < PG_NSTATS) pg_site_stat(sstats + site * 8, 1, deg > 1, deg, 1, __popc(amask), wgt);
+        if (deg > 1) return PG_EVENT_RAW(c, evm, PGK_BANK, round, rec, astar, ta, tb, site, deg, 0);
     }
     return 0u;
 }
 
 __device__ __noinline__ u32 pg_coal_global(u32 round, u32 lane, u32 ekey, u32 gtid, PgCold& c, u32 evm,
-                                           u64* sstats, u32 active, u32 rec, u32 flat, u32 site) {
+                                           u64* sstats, u32 active, u32 rec, u32 flat, u32 site, u32 wgt = 1u) {
     const u32 seg = __match_any_sync(PG_FULL, ekey);
     const u32 amask = __ballot_sync(PG_FULL, active) & seg;
     const u32 w = active ? flat : 0u;
@@ -298,8 +304,9 @@ __device__ __noinline__ u32 pg_coal_global(u32 round, u32 lane, u32 ekey, u32 gt
     const u32 ta = __reduce_min_sync(seg, active ? gtid : PG_NEVER);
     const u32 tb = __reduce_max_sync(seg, active ? gtid : 0u);
     if (amask && lane == (u32)(__ffs(amask) - 1)) {
-        if (sstats && site < PG_NSTATS) pg_site_stat(sstats + site * 8, 2, sectors > ideal, sectors, ideal, __popc(amask));
-        if (sectors > ideal) return pg_event(c, evm, PGK_UNCOAL, round, rec, amin, ta, tb, site, sectors, ideal);
+        if (sstats && site < PG_NSTATS)
+            pg_site_stat(sstats + site * 8, 2, sectors > ideal, sectors, ideal, __popc(amask), wgt);
+        if (sectors > ideal) return PG_EVENT_RAW(c, evm, PGK_UNCOAL, round, rec, amin, ta, tb, site, sectors, ideal);
     }
     return 0u;
 }
@@ -775,6 +782,10 @@ __device__ __forceinline__ void pg_log_write_ms(PgC& C, PgT& t, PgCold& c, u32 c
 template <int A, bool RD, bool LOG>
 __device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
                                             u32 (&v)[PG_MS]) {
+#if PG_BANKCHK
+    t.evm |= pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, t.evm, ss, pe & (flat < PG_SH(A, size)),
+                            PG_ARR(A).rec_id, flat, site, t.nsv);
+#endif
     PG_S_LOOP v[_s] = 0u;
     if (!pe) return;
     const u32 rec = PG_ARR(A).rec_id;
@@ -805,6 +816,10 @@ __device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 template <int A, bool RDA = false>
 __device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat,
                                             const u32 (&val)[PG_MS], u32 site) {
+#if PG_BANKCHK
+    t.evm |= pg_bank_shared(C.round, t.lane, t.ekey, t.tlin, t.gtid, c, t.evm, ss, pe & (flat < PG_SH(A, size)),
+                            PG_ARR(A).rec_id, flat, site, t.nsv);
+#endif
     if (!pe) return;
     if (flat >= PG_SH(A, size)) {
 #if PG_OOBCHK
@@ -825,6 +840,10 @@ __device__ __forceinline__ void pg_xb_mark_ms(const PgT& t, u32 flat) {
 template <int A, bool RD, bool LOG>
 __device__ __forceinline__ void pg_ld_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
                                             u32 (&v)[PG_MS]) {
+#if PG_COALCHK
+    t.evm |= pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, t.evm, ss, pe & (flat < PG_ARR(A).size),
+                            PG_ARR(A).rec_id, flat, site, t.nsv);
+#endif
     PG_S_LOOP v[_s] = 0u;
     if (!pe) return;
     if (flat >= PG_ARR(A).size) {
@@ -848,6 +867,10 @@ __device__ __forceinline__ void pg_ld_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 template <int A, bool RDA = false>
 __device__ __forceinline__ void pg_st_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat,
                                             const u32 (&val)[PG_MS], u32 site) {
+#if PG_COALCHK
+    t.evm |= pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, t.evm, ss, pe & (flat < PG_ARR(A).size),
+                            PG_ARR(A).rec_id, flat, site, t.nsv);
+#endif
     if (!pe) return;
     if (flat >= PG_ARR(A).size) {
 #if PG_OOBCHK
@@ -861,6 +884,10 @@ __device__ __forceinline__ void pg_st_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 template <int A>
 __device__ __forceinline__ void pg_ld_gi_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
                                             u32 (&v)[PG_MS]) {
+#if PG_COALCHK
+    t.evm |= pg_coal_global(C.round, t.lane, t.ekey, t.gtid, c, t.evm, ss, pe & (flat < PG_ARR(A).size),
+                            PG_ARR(A).rec_id, flat, site, t.nsv);
+#endif
     PG_S_LOOP v[_s] = 0u;
     if (!pe) return;
     if (flat >= PG_ARR(A).size) {

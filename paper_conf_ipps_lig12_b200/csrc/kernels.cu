@@ -280,7 +280,7 @@ __global__ void __launch_bounds__(256) pg_seq_select(const PgWork* __restrict__ 
 // K2c: fold the per-item site statistics of the block-parallel pass into the
 // per-launch table, skipping seed groups that the sequential pass re-runs.
 __global__ void __launch_bounds__(128) pg_stats_reduce(const PgWork* __restrict__ items, const u64* item_stats,
-                                                       const u32* flags, u64* launch_stats, u32 max_sites) {
+                                                       u32* flags, u64* launch_stats, u32 max_sites) {
     const PgWork w = items[blockIdx.x];
     __shared__ u32 s_skip;
     if (threadIdx.x == 0) {
@@ -289,7 +289,12 @@ __global__ void __launch_bounds__(128) pg_stats_reduce(const PgWork* __restrict_
         s_skip = f;
     }
     __syncthreads();
-    if (s_skip) return;
+    if (s_skip) {
+        // the sequential pass recomputes this item's statistics: make it re-run every seed of
+        // the item (a multi-seed item holds several whole one-seed sequential items)
+        for (u32 i = threadIdx.x; i < w.nseeds; i += blockDim.x) flags[w.inst0 + i] = 1u;
+        return;
+    }
     const u64* src = item_stats + (u64)w.item * max_sites * 8u;
     u64* dst = launch_stats + (u64)w.launch * max_sites * 8u;
     for (u32 i = threadIdx.x; i < max_sites * 8u; i += blockDim.x) {
@@ -519,7 +524,7 @@ cudaError_t seq_select(const PgWork* items, u32 n_items, const u32* flags, u32* 
     return cudaGetLastError();
 }
 
-cudaError_t stats_reduce(const PgWork* items, u32 n_items, const u64* item_stats, const u32* flags, u64* launch_stats,
+cudaError_t stats_reduce(const PgWork* items, u32 n_items, const u64* item_stats, u32* flags, u64* launch_stats,
                          u32 max_sites, cudaStream_t st) {
     if (!n_items) return cudaSuccess;
     pg_stats_reduce<<<n_items, 128, 0, st>>>(items, item_stats, flags, launch_stats, max_sites);
