@@ -1330,8 +1330,36 @@ __device__ __forceinline__ void pg_warp_merge(u32 pending, u64 key, u32 cnt_in, 
     key_out = lkey;
 }
 
+// Monotone 64-bit prefix of the X16 event order: (round, array, addr, tid_a) in 16 / 10 / 26 /
+// 12 bits, a field that does not fit saturates and zeroes the rest, so a <lex b implies
+// pg_pack(a) <= pg_pack(b).  Slots keep ~pg_pack of their minimum (atomicMax): a candidate
+// whose pack is larger cannot be the minimum and skips the lock - thousands of CTAs that
+// report events of one instance (one slot) no longer serialise on it.
+__device__ __forceinline__ u64 pg_pack(const u32* f) {
+    const u32 bits[4] = {16u, 10u, 26u, 12u};
+    u64 k = 0;
+    bool sat = false;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const u64 mx = (1ull << bits[i]) - 1ull;
+        u64 v = f[i];
+        if (sat) v = 0;
+        else if (v >= mx) { v = mx; sat = true; }
+        k = (k << bits[i]) | v;
+    }
+    return k;
+}
+// true when the slot already holds an event that precedes every event packing to `best`
+__device__ __forceinline__ bool pg_slot_skip(PgSlot* s, const u32* best) {
+    const u64 pk = ~pg_pack(best);
+    if (pk < *(volatile u64*)&s->pkey) return true;   // (pkey only grows: a stale read is safe)
+    atomicMax(&s->pkey, pk);
+    return false;
+}
+
 __device__ __noinline__ void pg_slot_update(PgSlot* s, u32 cnt, const u32* best) {
     atomicAdd(&s->count, (u64)cnt);
+    if (pg_slot_skip(s, best)) return;
     while (atomicCAS(&s->lock, 0u, 1u) != 0u) {
     }
     __threadfence();
@@ -1423,6 +1451,7 @@ struct PgFlushEntryMs {
 __device__ __noinline__ void pg_slot_update_ms(PgSlot* s0, u64 step, u32 nsv, u32 cnt, const u32* f6,
                                                const u32 (*v)[2]) {
     for (u32 q = 0; q < nsv; q++) atomicAdd(&s0[q * step].count, (u64)cnt);
+    if (pg_slot_skip(s0, f6)) return;
     while (atomicCAS(&s0->lock, 0u, 1u) != 0u) {
     }
     __threadfence();
@@ -1599,6 +1628,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 sl->count = 0;
                 sl->has = 0;
                 sl->lock = 0;
+                sl->pkey = 0;
             }
             if (threadIdx.x == 0u) P.inst_cnt[pg_sW.inst0 + ms] = 0ull;   // counted again below
         }

@@ -435,6 +435,7 @@ __global__ void __launch_bounds__(256) pg_reset_flagged(const u32* flags, u32 n_
         s[k].count = 0ull;
         s[k].lock = 0u;
         s[k].has = 0u;
+        s[k].pkey = 0ull;
     }
 }
 

@@ -75,6 +75,8 @@ struct PgSlot {
     u64 count;
     u32 lock, has;
     u32 f[8];  // round, array, addr, tid_a, tid_b, site, val_a, val_b
+    u64 pkey;  // ~(packed prefix of f) of the minimum event, maximised atomically (0: none):
+               // a candidate whose packed prefix is larger skips the lock (pg_pack)
 };
 
 struct PgParams {
