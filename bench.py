@@ -51,7 +51,9 @@ WORKLOADS = {
            "n <= 16", 64, 11, lambda W, s: W.c4("rand", s) + W.c4("range", s) + W.c4("bits")),
     "c5t": ("C5 transpose: naive vs 32x32 tiled transpose, N = 32..1024, %d seeds per GPU", 1250, 14,
             lambda W, s: [W.c5_transpose(n_seeds=s)]),
-    "c5m": ("C5 matmul: naive vs 32x32 tiled, N = 32..1024, K = 64, %d seeds per GPU", 1250, 10 * 64 + 10,
+    # matmul, K = 64: naive ~10 ops/k x 64 + 10 = 650 per thread in 1 round; tiled 2 load rounds (~14)
+    # + 2 compute rounds (~10 ops/k x 32) + a store round (~10) = ~678 over 5 rounds: (650 + 678) / 6
+    "c5m": ("C5 matmul: naive vs 32x32 tiled, N = 32..1024, K = 64, %d seeds per GPU", 1250, (650 + 678) // 6,
             lambda W, s: [W.c5_matmul(n_seeds=s)]),
 }
 WL = "c2"

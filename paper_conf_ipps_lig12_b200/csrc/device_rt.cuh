@@ -179,6 +179,7 @@ struct PgCold {     // per-emulated-thread state that lives in local memory
     u32 lvs[PG_WMAX][PG_MS];   // (see pg_lv_t)     // write-log values per seed (entries 1..)
     u32 ebv[PG_NK][PG_MS][2];    // per seed: (val_a, val_b) of the minimum event; fields 0..5 of
                                  // ebest are seed-independent (same accesses in every seed)
+    u64 epk[PG_NK];              // pg_pack of ebest[kind] (one 64-bit compare decides most events)
 #endif
 };
 
@@ -190,6 +191,25 @@ __device__ __forceinline__ bool pg_lex_less(const u32* a, const u32* b) {
     return false;
 }
 
+// Monotone 64-bit prefix of the X16 event order: (round, array, addr, tid_a) in 16 / 10 / 26 /
+// 12 bits, a field that does not fit saturates and zeroes the rest, so a <lex b implies
+// pg_pack(a) <= pg_pack(b).  Slots keep ~pg_pack of their minimum (atomicMax): a candidate
+// whose pack is larger cannot be the minimum and skips the lock - thousands of CTAs that
+// report events of one instance (one slot) no longer serialise on it.
+__device__ __forceinline__ u64 pg_pack(const u32* f) {
+    const u32 bits[4] = {16u, 10u, 26u, 12u};
+    u64 k = 0;
+    bool sat = false;
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+        const u64 mx = (1ull << bits[i]) - 1ull;
+        u64 v = f[i];
+        if (sat) v = 0;
+        else if (v >= mx) { v = mx; sat = true; }
+        k = (k << bits[i]) | v;
+    }
+    return k;
+}
 // Records an event of `kind`; `evm` is the caller's event mask (PgT::evm).  Returns the
 // kind's bit, which the caller ORs into its mask.
 __device__ __noinline__ u32 pg_event(PgCold& c, u32 evm, u32 kind, u32 round, u32 arr, u32 addr, u32 ta, u32 tb,
@@ -716,13 +736,16 @@ __device__ __noinline__ u32 pg_event_ms(PgCold& c, u32 evm, u32 kind, u32 round,
                                         u32 tb, u32 site, const u32* va, u32 vb) {
     const u32 e[6] = {round, arr, addr, ta, tb, site};
     const u32 has = (evm >> kind) & 1u;
+    const u64 pk = pg_pack(e);
     int cmp = -1;
     if (has) {
-        cmp = 0;
+        const u64 bp = c.epk[kind];
+        cmp = pk < bp ? -1 : pk > bp ? 1 : 0;   // (pg_pack is monotone: unequal packs decide)
         for (int i = 0; i < 6 && cmp == 0; i++)
             if (e[i] != c.ebest[kind][i]) cmp = e[i] < c.ebest[kind][i] ? -1 : 1;
     }
     if (cmp < 0) {
+        c.epk[kind] = pk;
         for (int i = 0; i < 6; i++) c.ebest[kind][i] = e[i];
         PG_S_LOOP { c.ebv[kind][_s][0] = va[_s]; c.ebv[kind][_s][1] = vb; }
     } else if (cmp == 0) {   // same access: the per-seed values decide (X16 lexicographic order)
@@ -1330,25 +1353,6 @@ __device__ __forceinline__ void pg_warp_merge(u32 pending, u64 key, u32 cnt_in, 
     key_out = lkey;
 }
 
-// Monotone 64-bit prefix of the X16 event order: (round, array, addr, tid_a) in 16 / 10 / 26 /
-// 12 bits, a field that does not fit saturates and zeroes the rest, so a <lex b implies
-// pg_pack(a) <= pg_pack(b).  Slots keep ~pg_pack of their minimum (atomicMax): a candidate
-// whose pack is larger cannot be the minimum and skips the lock - thousands of CTAs that
-// report events of one instance (one slot) no longer serialise on it.
-__device__ __forceinline__ u64 pg_pack(const u32* f) {
-    const u32 bits[4] = {16u, 10u, 26u, 12u};
-    u64 k = 0;
-    bool sat = false;
-#pragma unroll
-    for (int i = 0; i < 4; i++) {
-        const u64 mx = (1ull << bits[i]) - 1ull;
-        u64 v = f[i];
-        if (sat) v = 0;
-        else if (v >= mx) { v = mx; sat = true; }
-        k = (k << bits[i]) | v;
-    }
-    return k;
-}
 // true when the slot already holds an event that precedes every event packing to `best`
 __device__ __forceinline__ bool pg_slot_skip(PgSlot* s, const u32* best) {
     const u64 pk = ~pg_pack(best);
