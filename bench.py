@@ -319,14 +319,16 @@ def main():
     torch.cuda.synchronize()
     clocks.start()
     clocks.wait_first()
-    evs, all_runs = [], []
+    evs, all_runs, host_ms = [], [], []
     for k in range(args.steps):
         with torch.cuda.stream(stream):
             flush.fill_(1)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        h0 = time.perf_counter()
         e0.record(stream)
         all_runs.append(step(keys[k], cnts[k]))
         e1.record(stream)
+        host_ms.append(1000 * (time.perf_counter() - h0))
         evs.append((e0, e1))
     clocks.wait_sample(timeout=2.0)   # (the enqueued steps are still running: a sample under load)
     torch.cuda.synchronize()
@@ -346,6 +348,7 @@ def main():
             eval_ms += t["ms_eval"]
     if args.diag and rank == 0:
         print("device ms per step:", ["%.1f" % x for x in step_ms], file=sys.stderr)
+        print("host enqueue ms per step:", ["%.1f" % x for x in host_ms], file=sys.stderr)
     del all_runs
 
     # ---- end-to-end phase: the same steps through the C ABI, host launch lists in, records and
