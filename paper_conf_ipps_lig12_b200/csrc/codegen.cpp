@@ -577,7 +577,37 @@ struct Gen {
         }
         line("}");
     }
+    // ---------------------------------------------------------------- fuel (X19)
+    static bool has_kind(const Stmt* s, SK k) {
+        if (!s) return false;
+        if (s->kind == k) return true;
+        for (const Stmt* x : s->seq)
+            if (has_kind(x, k)) return true;
+        return has_kind(s->body, k) || has_kind(s->other, k) || has_kind(s->init, k) ||
+               has_kind(s->step, k);
+    }
+    // The back-edge of a loop whose body passes its last top-level barrier on every
+    // path to the back-edge (no `continue` before that barrier), with no loop after
+    // the barrier or in the step, is the first back-edge of its round: the round began
+    // at that barrier.  Its fuel count (1) cannot exceed the limit, so only the
+    // counters advance (same counts as pg_tick; the check is dropped).
+    static bool first_backedge_of_round(const Stmt* s) {
+        const Stmt* b = s->body;
+        if (!b || has_kind(s->step, SK::Loop)) return false;
+        if (b->kind == SK::Sync) return true;
+        if (b->kind != SK::Seq) return false;
+        int last = -1;
+        for (size_t i = 0; i < b->seq.size(); i++)
+            if (b->seq[i]->kind == SK::Sync) last = (int)i;
+        if (last < 0) return false;
+        for (int i = 0; i < last; i++)
+            if (has_kind(b->seq[i], SK::Continue)) return false;
+        for (size_t i = last + 1; i < b->seq.size(); i++)
+            if (has_kind(b->seq[i], SK::Loop)) return false;
+        return true;
+    }
     void uniform_loop(const Stmt* s) {
+        const bool fuel_free = first_backedge_of_round(s);
         if (s->init) stmt(s->init);
         Loop L;
         L.id = s->loop;
@@ -597,9 +627,13 @@ struct Gen {
         body << "L" << L.cont_label << ":;\n";
         if (s->step) stmt(s->step);
         loops.pop_back();
-        line("pg_tick(C, t, c, t.live);");
-        line(inline_ ? "if (++C.ufuel > C.fuel) { t.live = 0u; goto PG_DONE; }"
-                     : "if (++C.ufuel > C.fuel) { t.live = 0u; return PG_END; }");
+        if (fuel_free) {
+            line("t.fuel += (t.live != 0u); ++C.ufuel;");
+        } else {
+            line("pg_tick(C, t, c, t.live);");
+            line(inline_ ? "if (++C.ufuel > C.fuel) { t.live = 0u; goto PG_DONE; }"
+                         : "if (++C.ufuel > C.fuel) { t.live = 0u; return PG_END; }");
+        }
         line("goto L" + std::to_string(head) + ";");
         body << "L" << L.exit_label << ":;\n";
     }

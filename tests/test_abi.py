@@ -121,3 +121,24 @@ def test_seed_oblivious_cases(pgvc, body, oblivious):
     text = ("kernel k(global in int a[n], global out int b[n], unsigned n) {\n"
             "  unsigned t = tid.x;\n  %s\n}\n" % body)
     assert pgvc.load_ir(text).seed_oblivious()[0] == oblivious
+
+
+@pytest.mark.parametrize("body,checked,elided", [
+    # the back-edge follows the body's last barrier: the first back-edge of its round
+    ("for (int i = 0; i < n; i++) { s[tid.x] = i; sync; }", 0, 1),
+    ("for (int i = 0; i < n; i++) { for (int j = 0; j < n; j++) s[tid.x] = j; sync; }", 1, 1),
+    # a loop between the last barrier and the back-edge can spend the round's fuel first
+    ("for (int i = 0; i < n; i++) { sync; for (int j = 0; j < n; j++) s[tid.x] = j; }", 2, 0),
+    # `continue` before the barrier reaches the back-edge without it
+    ("for (int i = 0; i < n; i++) { if (n > 3) continue; sync; }", 1, 0),
+    # no barrier: the loop may iterate within one round
+    ("for (int i = 0; i < n; i++) { s[tid.x] = i; }", 1, 0),
+])
+def test_fuel_check_elision(pgvc, body, checked, elided):
+    """X19 fuel: the generated back-edge keeps its limit check unless the back-edge
+    is provably the first of its round (codegen first_backedge_of_round)."""
+    src = "kernel k(global out int o[4], int n) { shared int s[bdim.x]; %s o[0] = 1; }" % body
+    text = pgvc.load_ir(src).source()
+    n_bodies = max(1, text.count(" seg(Frame& F") + text.count(" run(Frame& F"))
+    assert text.count("++C.ufuel > C.fuel") == checked * n_bodies
+    assert text.count("t.fuel += (t.live != 0u); ++C.ufuel;") == elided * n_bodies
