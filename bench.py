@@ -225,6 +225,9 @@ def main():
     ap.add_argument("--diag", action="store_true", help="print per-step enqueue / device / per-check times")
     ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS),
                     help="c2 (headline, BASELINE configs[1]); others: the remaining configs for reference")
+    ap.add_argument("--streams", type=int, default=1,
+                    help="streams the independent pairs are spread over (0: one per pair; default 1: one stream, "
+                         "DESIGN.md §6 'Concurrent pairs')")
     ap.add_argument("--seeds", type=int, default=0, help="seeds per GPU (default: the workload's)")
     args = ap.parse_args()
     global WL, SEEDS_PER_GPU, OPS_PER_INSTANCE
@@ -259,8 +262,12 @@ def main():
                 from paper_conf_ipps_lig12_b200 import workloads as W
                 irs[name] = pgvc.load_ir(W.subject(name))
     stream = torch.cuda.Stream()
-    first_key = torch.empty(11, dtype=torch.int64, device="cuda")
-    counts = torch.empty(16, dtype=torch.int64, device="cuda")
+    # the pairs are independent checks: with --streams S > 1 they are spread over S side
+    # streams forked from and joined back into `stream` (each pair has its own key/count rows)
+    n_side = args.streams if args.streams > 0 else len(wls)
+    side = [torch.cuda.Stream() for _ in range(n_side)] if n_side > 1 else [stream]
+    pair_keys = torch.empty(len(wls), 11, dtype=torch.int64, device="cuda")
+    pair_counts = torch.empty(len(wls), 16, dtype=torch.int64, device="cuda")
     step_keys = torch.empty(11, dtype=torch.int64, device="cuda")
     step_counts = torch.zeros(16, dtype=torch.int64, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
@@ -268,18 +275,24 @@ def main():
     def step(keys_out, counts_out):
         """One pass of the whole path over the workload (enqueue only): H1..H8 per pair, H9 at the end."""
         runs = []
+        fork = torch.cuda.Event()
+        fork.record(stream)
+        for i, w in enumerate(wls):
+            st = side[i % len(side)]
+            if st is not stream and i < len(side):
+                st.wait_event(fork)
+            # weak scaling: 64 seeds per GPU, seeds j = rank, rank + N, ... of a 64 x N seed space
+            ns = SEEDS_PER_GPU * world if w.input_mode != 1 else w.n_seeds   # exhaustive 0/1 sets are fixed
+            sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=ns, rank=rank, world=world,
+                            input_mode=w.input_mode, input_range=w.input_range,
+                            checks=w.checks, stream=st.cuda_stream, first_key=pair_keys[i], counts=pair_counts[i])
+            runs.append(pgvc.check_equiv(irs[w.src], irs[w.tgt], sp))
         with torch.cuda.stream(stream):
-            keys_out.fill_(2 ** 63 - 1)
-            counts_out.zero_()
-            for w in wls:
-                # weak scaling: 64 seeds per GPU, seeds j = rank, rank + N, ... of a 64 x N seed space
-                ns = SEEDS_PER_GPU * world if w.input_mode != 1 else w.n_seeds   # exhaustive 0/1 sets are fixed
-                sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=ns, rank=rank, world=world,
-                                input_mode=w.input_mode, input_range=w.input_range,
-                                checks=w.checks, stream=stream.cuda_stream, first_key=first_key, counts=counts)
-                runs.append(pgvc.check_equiv(irs[w.src], irs[w.tgt], sp))
-                torch.minimum(keys_out, first_key, out=keys_out)
-                counts_out.add_(counts)
+            for st in side:
+                if st is not stream:
+                    stream.wait_stream(st)
+            torch.amin(pair_keys, 0, out=keys_out)
+            torch.sum(pair_counts, 0, out=counts_out)
             distributed.reduce_summary(keys_out, counts_out)   # H9: the only cross-GPU traffic
         return runs
 
@@ -349,6 +362,7 @@ def main():
     if args.diag and rank == 0:
         print("device ms per step:", ["%.1f" % x for x in step_ms], file=sys.stderr)
         print("host enqueue ms per step:", ["%.1f" % x for x in host_ms], file=sys.stderr)
+        print("step keys/counts:", keys[-1].tolist(), cnts[-1].tolist(), file=sys.stderr)
     del all_runs
 
     # ---- end-to-end phase: the same steps through the C ABI, host launch lists in, records and
@@ -372,12 +386,19 @@ def main():
     sm_max = clk.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
     alu_peak = SM_COUNT * ALU_LANES_PER_SM_CLK * sm_max * 1e6
     per_gpu_inst = inst_total / world
-    achieved_ops = per_gpu_inst * OPS_PER_INSTANCE / (eval_ms / 1000.0) if eval_ms else None
+    # K2 time: with one stream, the sum of the evaluation launches' durations (CUDA events around
+    # each); with the pairs on concurrent streams those launches overlap each other and the other
+    # kernels, so a launch's duration is no longer the kernel's own - the whole device step time is
+    # used instead (a lower bound on K2's achieved rate: it also covers K1/K2b/K3/K4)
+    k2_basis = "k2_launches" if len(side) == 1 else "whole_step"
+    k2_s = eval_ms / 1000.0 if len(side) == 1 else dev_ms / 1000.0
+    achieved_ops = per_gpu_inst * OPS_PER_INSTANCE / k2_s if k2_s else None
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "config": {"workload": workload_desc(), "seeds_per_gpu": SEEDS_PER_GPU, "l2": "flushed between steps",
+                   "streams": len(side),
                    "parallelism": "dp%d over seeds" % world},
         "roofline": {"bound": "alu", "achieved": achieved_ops / 1e12 if achieved_ops else None,
                      "peak": alu_peak / 1e12, "unit": "Tops/s (int32, algorithmic IR ops)",
@@ -385,7 +406,7 @@ def main():
                      "traffic": ncu_profile().get("bytes_per_launch"),
                      "ncu_issue_active_pct": ncu_profile().get("issue_active_pct_time_weighted"),
                      "kernel": "pgk_eval (K2)", "ops_per_instance": OPS_PER_INSTANCE,
-                     "k2_ms_per_step": eval_ms / args.steps,
+                     "k2_ms_per_step": eval_ms / args.steps, "time_basis": k2_basis, "streams": len(side),
                      "peak_source": "148 SM x 64 int32 lanes/clk x sm_max_mhz (DESIGN.md §6)"},
         "e2e": {"value": e2e, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
                 "d2h_bytes_per_step": d2h // args.steps},

@@ -101,6 +101,35 @@ def test_c2_pairs_reduced_space(env, oracle, W, pair):
     assert_same(ref, recs, summ)
 
 
+def test_c2_pairs_concurrent_streams(env, oracle, W):
+    """bench.py's launch configuration: the seven C2 pairs enqueued together, one stream
+    each (forked from and joined into one stream), each pair writing its own key/count
+    rows; every pair must still equal the oracle."""
+    pgvc, torch = env
+    ws = W.c2(n_seeds=3, max_log_n=9, max_log_b=9)
+    main = torch.cuda.current_stream()
+    side = [torch.cuda.Stream() for _ in ws]
+    keys = torch.empty(len(ws), 11, dtype=torch.int64, device="cuda")
+    cnts = torch.empty(len(ws), 16, dtype=torch.int64, device="cuda")
+    fork = torch.cuda.Event()
+    fork.record(main)
+    runs = []
+    for i, w in enumerate(ws):
+        side[i].wait_event(fork)
+        sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=3, checks=w.checks, stream=side[i].cuda_stream,
+                        first_key=keys[i], counts=cnts[i])
+        runs.append(pgvc.check_equiv(ir(pgvc, W.subject(w.src)), ir(pgvc, W.subject(w.tgt)), sp))
+    for st in side:
+        main.wait_stream(st)
+    torch.cuda.synchronize()
+    for i, (w, run) in enumerate(zip(ws, runs)):
+        recs, summ = run.collect(cap=1 << 20)
+        ref = oracle.check(W.subject(w.src), W.subject(w.tgt), w.launch_src, w.launch_tgt, n_seeds=3,
+                           checks=w.checks, cap=1 << 20)
+        assert_same(ref, recs, summ)
+        assert cnts[i][0].item() == ref["counts"][0]
+
+
 def test_c2_full_size_launches(env, oracle, W):
     # BASELINE sizes: N = 2^16 with B = 1, 32, 1024, one seed each (oracle computes these one by one)
     for src, tgt in (("reduce0", "reduce6"), ("reduce2", "reduce2_obo")):
