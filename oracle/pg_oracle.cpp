@@ -1164,10 +1164,21 @@ struct Exec {
     std::vector<Thread> th;
     std::map<Cell, std::set<uint32_t>> readers;   /* this round: cell -> reader tlin */
     std::vector<Access> accesses;                 /* this round */
-    /* VC-literal history: every committed write log of every earlier round
-       (shared: this block; global: this instance), per thread */
-    struct Hist { uint32_t block, round; std::vector<std::vector<WEntry>> logs; };
+    /* VC-literal history (L521-L522, L598-L599, L709-L712): the state at the start of
+       every round of this instance - each thread's registers and pc, the block's shared
+       memory and the global memory - so that the guard p(s) and address e(s) of every
+       write of thread s in that round can be re-evaluated on their own, independently of
+       the write logs, commits and ownership tables of the execution being checked. */
+    struct Hist {
+        uint32_t block, round;
+        std::vector<Thread> start;
+        std::vector<std::vector<uint32_t>> sval, gval;
+        std::vector<std::vector<uint8_t>> swritten;
+        std::vector<std::vector<Cell>> wset;   /* per thread: cells it writes (lazily re-evaluated) */
+        bool evaluated = false;
+    };
     std::vector<Hist> hist;
+    const Hist* shadow = nullptr;   /* non-null while re-evaluating a thread of that round */
 
     Exec(const Config& c, const KInfo& ki, const Launch& l, uint64_t sd, uint32_t li, uint32_t si, uint32_t ki_,
          Slot* sl, Results& r)
@@ -1176,6 +1187,7 @@ struct Exec {
 
     void event(int kind, uint32_t round, uint32_t arr, uint32_t addr, uint32_t ta, uint32_t tb, uint32_t site,
                uint32_t va, uint32_t vb) {
+        if (shadow) return;   /* re-evaluation for the VC-literal check reports nothing */
         Ev e;
         e.f[0] = round; e.f[1] = arr; e.f[2] = addr; e.f[3] = ta; e.f[4] = tb; e.f[5] = site; e.f[6] = va; e.f[7] = vb;
         slots[kind].add(e);
@@ -1220,36 +1232,77 @@ struct Exec {
     }
 
     void record_access(const Thread& t, int site, int a, uint32_t addr) {
-        if (!(cfg.checks & (CHK_BANK | CHK_COALESCE))) return;
+        if (shadow || !(cfg.checks & (CHK_BANK | CHK_COALESCE))) return;
         Access ac;
         ac.tlin = t.tlin; ac.gtid = t.gtid; ac.site = site; ac.arr = a; ac.addr = addr;
         for (int l : K.site_loops[(size_t)site]) ac.iter.push_back(t.loopctr[(size_t)l]);
         accesses.push_back(ac);
     }
     void mark_xb(int a, uint32_t addr) {
-        if (K.arrs[(size_t)a].space != SP_GLOBAL) return;
+        if (shadow || K.arrs[(size_t)a].space != SP_GLOBAL) return;
         auto& f = gfirst_blk[(size_t)a];
         if (f[addr] == 0) f[addr] = cur_block + 1;
         glast_blk[(size_t)a][addr] = cur_block + 1;
     }
 
-    /* VC-literal writer of cell c read in the current round: enumerate every
-       thread s of every earlier round (latest first) and test "s wrote c"
-       literally; returns (found, block, round, min writer tlin). */
+    /* Fig. 2 instantiation (L582-L599): for every thread s of round H, evaluate its
+       segment alone from the round-start state - the values of its guards p(s) and write
+       addresses e(s) - and keep the cells it writes.  Reads see the round-start memory
+       plus s's own earlier writes (X3), exactly as in the paper's per-thread CA maps. */
+    void literal_write_sets(Hist& H) {
+        if (H.evaluated) return;
+        const uint32_t blk = cur_block, b0 = bid[0], b1 = bid[1], b2 = bid[2];
+        cur_block = H.block;
+        bid[0] = H.block % L.gdim[0];
+        bid[1] = (H.block / L.gdim[0]) % L.gdim[1];
+        bid[2] = H.block / (L.gdim[0] * L.gdim[1]);
+        shadow = &H;
+        H.wset.assign(H.start.size(), {});
+        for (size_t s = 0; s < H.start.size(); s++) {
+            if (H.start[s].exited) continue;
+            Thread t = H.start[s];
+            t.wlog.clear();
+            run_thread(t);
+            for (const WEntry& w : t.wlog) H.wset[s].push_back(w.c);
+        }
+        shadow = nullptr;
+        cur_block = blk;
+        bid[0] = b0; bid[1] = b1; bid[2] = b2;
+        H.evaluated = true;
+    }
+
+    /* VC-literal writer of cell c read in the current round: for every earlier round
+       (latest first; shared cells: this block's rounds, global cells: every block run so
+       far) enumerate all threads s and test p(s) ∧ c = e(s) on the re-evaluated maps
+       (L521-L522, L709-L712); returns (found, block, round, min writer tlin).  More than one
+       s is exactly a WW race (L517-L518). */
     bool vc_literal_writer(const Cell& c, bool global, uint32_t& wb, uint32_t& wr, uint32_t& wt) {
-        for (size_t h = hist.size(); h-- > 0;) {
-            const Hist& H = hist[h];
+        for (size_t h = hist.size() - 1; h-- > 0;) {   /* (the last entry is the current round) */
+            Hist& H = hist[h];
             if (!global && H.block != cur_block) continue;
+            literal_write_sets(H);
             std::vector<uint32_t> S;
-            for (uint32_t s = 0; s < (uint32_t)H.logs.size(); s++)
-                for (const WEntry& w : H.logs[s])
-                    if (w.c == c) S.push_back(s);
+            for (uint32_t s = 0; s < (uint32_t)H.wset.size(); s++)
+                for (const Cell& w : H.wset[s])
+                    if (w == c) S.push_back(s);
             if (!S.empty()) {
                 wb = H.block; wr = H.round; wt = *std::min_element(S.begin(), S.end());
                 return true;
             }
         }
         return false;
+    }
+
+    /* a load while re-evaluating a thread for the VC-literal check: round-start memory */
+    uint32_t shadow_load(Thread& t, int a, uint32_t f) {
+        const Arr& A = K.arrs[(size_t)a];
+        if (f >= size[(size_t)a]) return poison(a, f);
+        Cell c{a, f};
+        for (const WEntry& w : t.wlog)
+            if (w.c == c) return w.val;
+        if (A.space == SP_GLOBAL) return shadow->gval[(size_t)a][f];
+        const size_t li = (size_t)A.local_index;
+        return shadow->swritten[li][f] ? shadow->sval[li][f] : poison(a, f);
     }
 
     uint32_t load(Thread& t, const Expr* e) {
@@ -1265,6 +1318,7 @@ struct Exec {
             }
             return t.parr[(size_t)A.local_index][f];
         }
+        if (shadow) return shadow_load(t, a, f);
         if (f >= size[(size_t)a]) {
             uint32_t pv = poison(a, f);
             if (cfg.checks & CHK_OOB) event(K_OOB, cur_round, rec_arr_id(a), f, t.gtid, NONE32, (uint32_t)e->site, pv, 0);
@@ -1579,6 +1633,12 @@ struct Exec {
             for (;;) {
                 readers.clear();
                 for (uint32_t i = 0; i < T; i++) th[i].wlog.clear();
+                if (cfg.vcliteral) {   /* round-start state for the literal re-evaluation */
+                    Hist H;
+                    H.block = b; H.round = cur_round; H.start = th; H.sval = sval; H.swritten = swritten;
+                    H.gval = gval;
+                    hist.push_back(std::move(H));
+                }
                 /* natural order, L384-L389 */
                 for (uint32_t i = 0; i < T; i++)
                     if (!th[i].exited) run_thread(th[i]);
@@ -1606,11 +1666,6 @@ struct Exec {
                             sn.cells.push_back(swritten[li][i] ? ((1ull << 32) | sval[li][i]) : 0ull);
                         res.snaps[kernel_idx].push_back(std::move(sn));
                     }
-                }
-                if (cfg.vcliteral) {
-                    Hist H; H.block = b; H.round = cur_round;
-                    for (uint32_t i = 0; i < T; i++) H.logs.push_back(th[i].wlog);
-                    hist.push_back(std::move(H));
                 }
                 bool any = false;
                 for (uint32_t i = 0; i < T; i++) any |= !th[i].exited;
