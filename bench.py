@@ -410,6 +410,8 @@ def main():
                      "peak_source": "148 SM x 64 int32 lanes/clk x sm_max_mhz (DESIGN.md §6)"},
         "e2e": {"value": e2e, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
                 "d2h_bytes_per_step": d2h // args.steps},
+        "step_ms": {"median": statistics.median(step_ms), "min": min(step_ms), "max": max(step_ms),
+                    "host_enqueue_median": statistics.median(host_ms)},
         "gpu_launches": launches // args.steps * args.steps,
         "clocks": clk,
     }

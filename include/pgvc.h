@@ -50,7 +50,11 @@ enum {
 enum { PG_IN_RAND32 = 0, PG_IN_BITS01 = 1, PG_IN_RANGE = 2 };                 /* X8 */
 enum { PG_CHK_EQUIV = 1, PG_CHK_RACE = 2, PG_CHK_OOB = 4, PG_CHK_BANK = 8, PG_CHK_COALESCE = 16,
        PG_CHK_DATAFLOW = 32, /* record the writer of every read (H5); evaluates blocks in bid order */
-       PG_CHK_LOCKSTEP = 64  /* pg_check_equiv: compare the kernels' shared state round by round */ };
+       PG_CHK_LOCKSTEP = 64, /* pg_check_equiv: compare the kernels' shared state round by round */
+       PG_CHK_OPCOUNT = 128  /* measurement: count the IR integer operations the kernels execute (each
+                                unary / binary / logical / select / min / max node and two per extra array
+                                dimension, under the thread's predicate) into d_counts[13]; exact
+                                single-seed passes */ };
 enum { PG_LOCK_ROUNDS = 32 };   /* rounds of every block the lock-step comparison covers */
 enum { PG_BANKS_32 = 0, PG_BANKS_16_HALFWARP = 1 };                             /* X9 */
 enum {                                                                          /* X17 */
@@ -84,7 +88,8 @@ typedef struct {
     void *cuda_stream;                         /* borrowed cudaStream_t (0 = legacy default stream) */
     int64_t *d_first_key;                      /* borrowed device int64[11]: [0] min failing key, [1+k] min key of kind k; INT64_MAX = none */
     int64_t *d_counts;                         /* borrowed device int64[16]: [0] instances (X19), [1+k] events of kind k,
-                                                  [11] records, [12] failing (launch, seed) instances */
+                                                  [11] records, [12] failing (launch, seed) instances,
+                                                  [13] IR operations executed (PG_CHK_OPCOUNT only) */
 } pg_space;
 
 /* One counterexample record (X16): the minimum event of its (launch, seed,
@@ -104,6 +109,7 @@ typedef struct {
     uint32_t first_seed_idx;
     uint64_t per_kind[PG_N_KINDS];
     int64_t first_key_kind[PG_N_KINDS];
+    uint64_t ir_ops;           /* d_counts[13]: IR operations executed (PG_CHK_OPCOUNT runs) */
 } pg_summary;
 
 /* Parse, check and code-generate one kernel (the IR of DESIGN.md §4; the
@@ -139,10 +145,12 @@ int pg_check_banks(const pg_ir *k, const pg_space *sp, pg_run **out);
  * than the available values is PG_E_ARG. */
 int pg_check_property(const pg_ir *k, const pg_ir *post, const pg_space *sp, pg_run **out);
 
-/* Synchronise the run's stream, copy the first min(*n_written, cap, max_cex)
- * records (canonical key order; the run keeps at most pg_space.max_cex, 0 =
- * 2^20) into buf, report how many exist in *n_written (may exceed both caps),
- * and fill *sum (may be NULL) from d_first_key / d_counts as they are now. */
+/* Synchronise the run's stream, copy the first min(*n_written, cap, max_cex) of the
+ * run's OWN records (canonical key order; the run keeps at most pg_space.max_cex,
+ * 0 = 2^20) into buf, report how many this run produced in *n_written (may exceed both
+ * caps; never the cross-rank total), and fill *sum (may be NULL) from d_first_key /
+ * d_counts as they are now - after an all_reduce these are the global summary, so
+ * sum->n_records may exceed *n_written. */
 int pg_collect_cex(pg_run *r, pg_cex *buf, size_t cap, size_t *n_written, pg_summary *sum);
 
 /* Per-site bank/coalescing statistics of a run: uint64
@@ -188,8 +196,24 @@ int pg_ir_compile(const pg_ir *k, uint32_t bits, uint32_t checks, uint32_t bank_
 
 /* Device time of the run's evaluation kernels and of the whole check (CUDA
  * events on the run's stream, ms), the number of CUDA kernels it launched and
- * the host->device bytes it copied (launch tables, work lists). */
+ * the host->device bytes it copied (launch tables).  A check whose plan was seen before
+ * replays a captured CUDA graph of its body (PGVC_GRAPH=0 disables), so repeated checks
+ * enqueue a handful of operations and allocate only their record list. */
 int pg_run_timing(pg_run *r, float *ms_eval, float *ms_total, uint32_t *n_launches, uint64_t *h2d_bytes);
+
+/* Start and end (ms) of each of the run's evaluation-kernel launches, as pairs in buf[2i],
+ * buf[2i+1], relative to ref_event (a cudaEvent_t recorded before the check, e.g. the
+ * caller's step-start event; NULL = the run's first enqueued operation).  The union of
+ * these intervals is the evaluation kernel's busy time when launches overlap (the two
+ * kernels of a pair run on parallel branches).  *n = number of launches; at most cap pairs
+ * are written.  Synchronises the run's stream. */
+int pg_run_intervals(pg_run *r, void *ref_event, float *buf, size_t cap, size_t *n);
+
+/* Measurement utility (not part of the method; the K2 roofline denominator, SURVEY.md
+ * §8(d)): integer ops/s the current device sustains on `stream` for [0] LOP3 chains (alu
+ * pipe), [1] IMAD chains (fma pipe), [2] both alternating (the two pipes together).
+ * ~50 ms of GPU time; PG_E_CUDA without a device. */
+int pg_measure_int32_peak(void *stream, double ops_per_s[3]);
 
 const char *pg_last_error(void);
 void pg_ir_free(pg_ir *k);

@@ -117,6 +117,7 @@ struct Gen {
     uint32_t mask;
     std::ostringstream body;
     int ntmp = 0, nlabel = 0, nsync = 0;
+    std::vector<uint32_t> sync_sites_;   // site of each seg() resume point, in order
 
     struct Loop {
         int id;
@@ -254,6 +255,7 @@ struct Gen {
     // reader stamps for this load site
     bool stamps_needed(const Node* n) const {
         if (!reader_tracked(n->ref)) return false;
+        if (K.div_barrier) return true;   // (threads of one round may have entered from different barriers)
         auto it = seg_ld_.find(n);
         if (it == seg_ld_.end()) return true;
         for (const Stmt* b : it->second)
@@ -309,6 +311,10 @@ struct Gen {
     }
 
     // ---------------------------------------------------------------- expressions
+    // PG_CHK_OPCOUNT: count one IR integer operation executed under predicate pr
+    void opc(const std::string& pr, int n = 1) {
+        if (O.checks & 128) line("t.ops += " + std::to_string(n) + "u * (u32)(" + pr + ");");
+    }
     std::string flat_index(const Node* n, int arr, const std::string& pr) {
         std::vector<std::string> iv;
         for (const Node* k : n->kids) iv.push_back(ex(k, pr));
@@ -321,10 +327,19 @@ struct Gen {
             else if (a.space == SHARED) dim = "PG_SH(" + std::to_string(arr) + ", d" + std::to_string(k) + ")";
             else dim = "pg_sL.arr[" + std::to_string(arr) + "].d" + std::to_string(k);
             line(f + " = " + f + " * " + dim + " + " + iv[k] + ";");
+            opc(pr, 2);   // (row-major flattening: a multiply and an add per extra dimension)
         }
         return f;
     }
     std::string ex(const Node* n, const std::string& pr) {
+        switch (n->kind) {
+        case NK::Neg: case NK::BitNot: case NK::LogNot: case NK::Bin: case NK::LAnd: case NK::LOr:
+        case NK::Select: case NK::Min: case NK::Max:
+            opc(pr);
+            break;
+        default:
+            break;
+        }
         switch (n->kind) {
         case NK::Lit: return hex(n->lit & mask);
         case NK::Var: return "F.v" + std::to_string(n->ref);
@@ -498,16 +513,19 @@ struct Gen {
                  std::to_string(a.slot) + "[_i] = 0u; }");
             return;
         }
+        // (a kernel with a barrier under thread-dependent control runs every branch as a
+        // per-thread branch: each thread stops at its own barrier, X18)
         case SK::If:
-            if (s->uniform) uniform_if(s);
+            if (s->uniform || K.div_barrier) uniform_if(s);
             else predicated_if(s);
             return;
         case SK::Loop:
-            if (s->uniform) uniform_loop(s);
+            if (s->uniform || K.div_barrier) uniform_loop(s);
             else predicated_loop(s);
             return;
         case SK::Sync: {
             int k = ++nsync;
+            if (!inline_) sync_sites_.push_back((uint32_t)s->site);
             if (inline_) {   // end this round in place; stop when every thread has exited
                 line("if (!pg_round_end<PgK, false>(C, t, c, ar)) return;");
                 return;
@@ -694,6 +712,7 @@ struct Gen {
         // `run` (a whole block, rounds ended in place)
         auto emit = [&](bool inl) {
             ntmp = nlabel = nsync = 0;
+            sync_sites_.clear();
             body.str("");
             preds.clear();
             loops.clear();
@@ -710,6 +729,7 @@ struct Gen {
         };
         const std::string seg_body = emit(false);
         const int seg_nsync = nsync;
+        const std::vector<uint32_t> seg_sites = sync_sites_;
         const std::string run_body = emit(true);
         std::ostringstream o;
         o << "#define PG_BITS " << O.bits << "\n";
@@ -721,6 +741,8 @@ struct Gen {
         o << "#define PG_DATAFLOW " << ((O.checks & 32) ? 1 : 0) << "\n";
         o << "#define PG_LOCKSTEP " << ((O.checks & 64) ? 1 : 0) << "\n";
         o << "#define PG_FAST " << (O.fast ? 1 : 0) << "\n";
+        o << "#define PG_DIVBAR " << (K.div_barrier ? 1 : 0) << "\n";
+        o << "#define PG_OPCOUNT " << ((O.checks & 128) ? 1 : 0) << "\n";
         o << "#define PG_WMAX " << O.wmax << "\n";
         o << "#define PG_MS " << (ms() ? O.ms : 1u) << "\n";
         o << "#define PG_NSTATS " << std::max<size_t>(1, K.sites.size()) << "\n";
@@ -788,6 +810,11 @@ struct Gen {
             }
         }
         o << "  }\n";
+        // site id of the barrier a seg() return value (resume point k >= 1) stands for (X18 records)
+        o << "  static __device__ __forceinline__ u32 sync_site(u32 k) {\n    switch (k) {\n";
+        for (size_t k = 0; k < seg_sites.size(); k++)
+            o << "      case " << (k + 1) << "u: return " << seg_sites[k] << "u;\n";
+        o << "      default: return PG_NEVER;\n    }\n  }\n";
         o << "  static __device__ __forceinline__ u32 seg(Frame& F, PgC& C, PgT& t, PgCold& c, u64* ss, u32 resume) {\n";
         o << "    switch (resume) {\n      case 0u: goto R0;\n";
         for (int k = 1; k <= seg_nsync; k++) o << "      case " << k << "u: goto R" << k << ";\n";

@@ -30,6 +30,12 @@
 #ifndef PG_FAST
 #define PG_FAST 0
 #endif
+#ifndef PG_OPCOUNT
+#define PG_OPCOUNT 0   // PG_CHK_OPCOUNT: count executed IR operations (measurement variant)
+#endif
+#ifndef PG_DIVBAR
+#define PG_DIVBAR 0    // a barrier under thread-dependent control: per-thread resume points (X18)
+#endif
 #define PG_MSX (PG_MS > 1 && !PG_FAST)
 #define PG_S_LOOP _Pragma("unroll") for (u32 _s = 0; _s < (u32)PG_MS; _s++)
 
@@ -159,6 +165,9 @@ struct PgT {        // hot per-emulated-thread state (kept in registers)
     u32 fuel;
     u32 sg;         // byte offset of this instance's shared region in pg_dsmem
     u32 nsv;        // multi-seed lanes: seeds of this lane's group (<= PG_MS)
+#if PG_OPCOUNT
+    u32 ops;        // IR integer operations this thread executed (PG_CHK_OPCOUNT)
+#endif
     u64 seed;
     u32* arena;     // this instance's kernel arena
     const u32* input;
@@ -1579,6 +1588,46 @@ __device__ __forceinline__ u32 pg_init_value(const PgParams& P, u64 seed, u32 gi
     return v & P.mask;
 }
 
+#if PG_DIVBAR
+// X18 at round end: the barrier sites the live threads of each emulated block wait at.
+// Two or more distinct sites -> one BARRIER_DIV event: (lowest site, second-lowest site)
+// and the lowest thread waiting at each (gtid), in the order of DESIGN.md X16/X18.
+// dv: 4 words per group (s0, s1, t0, t1), all-ones between rounds.
+template <class K>
+__device__ __forceinline__ void pg_barrier_div(const PgC& C, PgT* T, PgCold* Cd, const u32* rsm, u32 V, u32 g,
+                                               u32 tl0, u32 inst_ok, bool warp_blocks, u32* dv_all) {
+    u32* dv = dv_all + 4u * (inst_ok ? g : 0u);
+    u32 site[PG_VMAX];
+#pragma unroll
+    for (u32 v = 0; v < PG_VMAX; v++)
+        site[v] = (v < V && inst_ok && T[v].live) ? K::sync_site(rsm[v]) : PG_NEVER;
+#define PG_DV_BAR() do { if (warp_blocks) __syncwarp(); else __syncthreads(); } while (0)
+#pragma unroll
+    for (u32 v = 0; v < PG_VMAX; v++)
+        if (site[v] != PG_NEVER) atomicMin(&dv[0], site[v]);
+    PG_DV_BAR();
+    const u32 s0 = inst_ok ? dv[0] : PG_NEVER;
+#pragma unroll
+    for (u32 v = 0; v < PG_VMAX; v++)
+        if (site[v] != PG_NEVER && site[v] != s0) atomicMin(&dv[1], site[v]);
+    PG_DV_BAR();
+    const u32 s1 = inst_ok ? dv[1] : PG_NEVER;
+    if (s1 != PG_NEVER) {
+#pragma unroll
+        for (u32 v = 0; v < PG_VMAX; v++) {
+            if (site[v] == s0) atomicMin(&dv[2], T[v].gtid);
+            else if (site[v] == s1) atomicMin(&dv[3], T[v].gtid);
+        }
+    }
+    PG_DV_BAR();
+    if (s1 != PG_NEVER && tl0 == 0u) PG_EVENT(T[0], Cd[0], PGK_BARRIER_DIV, C.round, PG_NEVER, 0u, dv[2], dv[3], s0, s1, 0u);
+    PG_DV_BAR();
+    if (inst_ok && tl0 == 0u) dv[0] = dv[1] = dv[2] = dv[3] = PG_NEVER;
+    PG_DV_BAR();
+#undef PG_DV_BAR
+}
+#endif
+
 template <class K>
 __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     __shared__ u32 s_flag;
@@ -1635,6 +1684,9 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 sl->pkey = 0;
             }
             if (threadIdx.x == 0u) P.inst_cnt[pg_sW.inst0 + ms] = 0ull;   // counted again below
+#if PG_OPCOUNT
+            if (threadIdx.x == 0u) P.op_cnt[pg_sW.inst0 + ms] = 0ull;
+#endif
         }
         __threadfence();
         __syncthreads();
@@ -1661,6 +1713,9 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
     sstats = nullptr;
 #endif
     for (u32 i = threadIdx.x; i < PG_PK; i += blockDim.x) s_grounds[i] = 0;
+#if PG_DIVBAR
+    for (u32 i = threadIdx.x; i < 4u * PG_PK; i += blockDim.x) s_grounds[PG_PK + i] = PG_NEVER;
+#endif
 
     PgC C;
     pg_set_step(C, 0u);
@@ -1713,6 +1768,9 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         t.evm = 0u;
         t.fl = 0u;
         t.live = ok;
+#if PG_OPCOUNT
+        t.ops = 0u;
+#endif
     }
     __syncthreads();
     const bool grid_1d = pg_sL.gdim[1] == 1u && pg_sL.gdim[2] == 1u;
@@ -1750,7 +1808,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         if (pg_sL.off_step0 != ~0ull && inst_ok && tl0 == 0u && blk_ok) T[0].arena[pg_sL.off_step0 + blk] = C.step0;
 #endif
         C.round = 0;
-#if PG_VMAX == 1
+#if PG_VMAX == 1 && !PG_DIVBAR
         {   // rounds inline: K::run ends each round at its barrier (pg_round_end)
             PgT& t = T[0];
             pg_set_step(C, C.step + 1u);
@@ -1762,6 +1820,11 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         }
 #else
         u32 resume = 0;
+#if PG_DIVBAR
+        u32 rsm[PG_VMAX];   // per-thread resume points: each thread resumes after its own barrier (X18)
+#pragma unroll
+        for (u32 v = 0; v < PG_VMAX; v++) rsm[v] = 0u;
+#endif
         for (;;) {
             pg_set_step(C, C.step + 1u);
             C.ufuel = 0;
@@ -1773,9 +1836,16 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 any_start |= T[v].live;
                 T[v].nlog = 0;
                 T[v].fuel = 0;
+#if PG_DIVBAR
+                if (T[v].live) rsm[v] = K::seg(F[v], C, T[v], Cd[v], sstats, rsm[v]);
+#else
                 r = K::seg(F[v], C, T[v], Cd[v], sstats, resume);
+#endif
             }
             alive_rounds += any_start;
+#if PG_DIVBAR
+            pg_barrier_div<K>(C, T, Cd, rsm, V, g, tl0, inst_ok, warp_blocks, s_grounds + PG_PK);
+#endif
             u32 any = 0;
 #if PG_FAST
             if (warp_blocks) __syncwarp();
@@ -1829,7 +1899,11 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
 #else
             const int more = warp_blocks ? __any_sync(PG_FULL, any) : __syncthreads_or((int)any);
 #endif
+#if PG_DIVBAR
+            if (!more) break;
+#else
             if (r == PG_END || !more) break;
+#endif
             resume = r;
         }
 #endif
@@ -1948,6 +2022,15 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             for (u32 i = 0; i < nsv; i++) atomicAdd(&P.inst_cnt[key + i], x);
         }
     }
+#if PG_OPCOUNT
+    {   // IR operations per batch-local instance (PG_CHK_OPCOUNT; one seed per group here)
+        u64 x = 0;
+#pragma unroll
+        for (u32 v = 0; v < PG_VMAX; v++)
+            if (v < V && inst_ok) x += T[v].ops;
+        if (x) atomicAdd(&P.op_cnt[pg_sW.inst0 + sb], x);
+    }
+#endif
 #if PG_BANKCHK || PG_COALCHK
     __syncthreads();
     if (P.site_stats) {

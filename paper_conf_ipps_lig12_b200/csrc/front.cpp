@@ -843,7 +843,7 @@ public:
             changed_ = false;
             grid_walk(K.body);
         } while (changed_);
-        K.grid_uniform_control = grid_control(K.body);
+        K.grid_uniform_control = grid_control(K.body) && !K.div_barrier;
     }
 
 private:
@@ -967,9 +967,7 @@ private:
         if (!s) return;
         switch (s->kind) {
         case SK::Sync:
-            if (!u)
-                throw FrontError(PG_E_TYPE, where(s->line, s->col) +
-                                                "barrier under thread-dependent control flow (DESIGN.md X18)");
+            if (!u) K.div_barrier = true;   // checked at run time (X18)
             break;
         case SK::Seq:
             for (const Stmt* c : s->seq) check_syncs(c, u);

@@ -100,6 +100,10 @@ struct Kernel {
     // depend on bid): emulated blocks with different bid share one round structure
     // and can run lock-step in one CTA
     bool grid_uniform_control = true;
+    // some `sync` sits under thread-dependent control flow: threads of a block may wait at
+    // different barriers, which the run-time check X18 reports (BARRIER_DIV).  Such kernels
+    // are compiled with per-thread branches and per-thread resume points (codegen.cpp)
+    bool div_barrier = false;
     Stmt* body = nullptr;
     std::vector<std::unique_ptr<Node>> node_pool;
     std::vector<std::unique_ptr<Stmt>> stmt_pool;

@@ -387,10 +387,13 @@ struct PgCexDev {
 };
 
 // K4c: write each instance's records at its scanned offset (slot order = key order).
+// The run's record count (its own records, before any cross-rank reduction of the counters)
+// goes to *total.
 __global__ void __launch_bounds__(256) pg_compact(const PgSlot* __restrict__ slots, u32 n_inst, u32 n_local,
-                                                  u32 rank, u32 world, const u64* offsets, PgCexDev* out,
-                                                  u64 cap) {
+                                                  u32 rank, u32 world, const u32* inst_nrec, const u64* offsets,
+                                                  PgCexDev* out, u64 cap, u64* total) {
     const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
+    if (inst == 0) *total = offsets[n_inst - 1] + inst_nrec[n_inst - 1];
     if (inst >= n_inst) return;
     const u32 li = inst / n_local, m = inst % n_local;
     const u32 sj = rank + m * world;
@@ -452,6 +455,35 @@ __global__ void __launch_bounds__(1024) pg_count_reduce(const u64* inst_cnt, u32
         for (u32 w = 0; w < (blockDim.x + 31u) / 32u; w++) t += part[w];
         atomicAdd(counts, t);
     }
+}
+
+// ------------------------------------------------------------------ INT32 peak microbenchmark
+// Measurement only (the roofline denominator of K2): 8 independent
+// chains per thread of LOP3 (alu pipe, mode 0), IMAD (fma pipe, mode 1) or both
+// alternating (mode 2), 16 x 8 = 128 integer ops per loop trip.  inline PTX keeps ptxas
+// from folding the chains; the result is stored only under a condition it cannot decide.
+template <int MODE>
+__global__ void __launch_bounds__(256) pg_int_peak(u32 iters, u32* sink) {
+    u32 a[8];
+    const u32 b = threadIdx.x * 0x9E3779B9u + blockIdx.x, c = (u32)clock() | 1u;
+#pragma unroll
+    for (int j = 0; j < 8; j++) a[j] = b + (u32)j * 0x85EBCA6Bu;
+    for (u32 i = 0; i < iters; i++) {
+#pragma unroll
+        for (int r = 0; r < 16; r++) {
+#pragma unroll
+            for (int j = 0; j < 8; j++) {
+                if (MODE == 0 || (MODE == 2 && (j & 1)))
+                    asm volatile("lop3.b32 %0, %0, %1, %2, 0x6A;" : "+r"(a[j]) : "r"(b), "r"(c));
+                else
+                    asm volatile("mad.lo.u32 %0, %0, %1, %2;" : "+r"(a[j]) : "r"(c), "r"(b));
+            }
+        }
+    }
+    u32 x = 0;
+#pragma unroll
+    for (int j = 0; j < 8; j++) x ^= a[j];
+    if (x == 0x1234567u && b == c) sink[threadIdx.x] = x;
 }
 
 }  // namespace
@@ -537,15 +569,27 @@ cudaError_t reset_counters(long long* first_key, long long* counts, cudaStream_t
     return cudaGetLastError();
 }
 
-cudaError_t summarize_compact(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, u32 banks_mode,
-                              u32* inst_nrec, u64* offsets, void* out, u64 cap, long long* first_key,
-                              long long* counts, cudaStream_t st) {
+cudaError_t summarize_scan(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, u32 banks_mode,
+                           u32* inst_nrec, u64* offsets, long long* first_key, long long* counts, cudaStream_t st) {
     if (!n_inst) return cudaSuccess;
     pg_summarize<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, banks_mode, inst_nrec,
                                                        first_key, counts);
     pg_scan<<<1, 1024, 0, st>>>(inst_nrec, offsets, n_inst);
-    pg_compact<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, offsets,
-                                                     (PgCexDev*)out, cap);
+    return cudaGetLastError();
+}
+
+cudaError_t compact(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, const u32* inst_nrec,
+                    const u64* offsets, void* out, u64 cap, u64* total, cudaStream_t st) {
+    if (!n_inst) return cudaSuccess;
+    pg_compact<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, inst_nrec, offsets,
+                                                     (PgCexDev*)out, cap, total);
+    return cudaGetLastError();
+}
+
+cudaError_t int_peak(int mode, u32 blocks, u32 iters, u32* sink, cudaStream_t st) {
+    if (mode == 0) pg_int_peak<0><<<blocks, 256, 0, st>>>(iters, sink);
+    else if (mode == 1) pg_int_peak<1><<<blocks, 256, 0, st>>>(iters, sink);
+    else pg_int_peak<2><<<blocks, 256, 0, st>>>(iters, sink);
     return cudaGetLastError();
 }
 

@@ -107,6 +107,7 @@ struct PgParams {
     u32 pad3;
     u32* flag_any;          // set when any instance of the batch is flagged; re-run passes with
                             // nothing flagged exit at once (nullptr: absent)
+    u64* op_cnt;            // PG_CHK_OPCOUNT: per batch-local instance, IR integer operations executed
 };
 
 // K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive

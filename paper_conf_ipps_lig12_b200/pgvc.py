@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(_HERE, "libpgvc.so")
 
 PG_OK, PG_E_ARG, PG_E_PARSE, PG_E_TYPE, PG_E_LIMIT, PG_E_CUDA, PG_E_OOM, PG_E_STATE = 0, -1, -2, -3, -4, -5, -6, -7
 IN_RAND32, IN_BITS01, IN_RANGE = 0, 1, 2
-CHK_EQUIV, CHK_RACE, CHK_OOB, CHK_BANK, CHK_COALESCE, CHK_DATAFLOW, CHK_LOCKSTEP = 1, 2, 4, 8, 16, 32, 64
+CHK_EQUIV, CHK_RACE, CHK_OOB, CHK_BANK, CHK_COALESCE, CHK_DATAFLOW, CHK_LOCKSTEP, CHK_OPCOUNT = 1, 2, 4, 8, 16, 32, 64, 128
 LOCK_ROUNDS = 32
 BANKS_32, BANKS_16_HALFWARP = 0, 1
 KINDS = ["BARRIER_DIV", "OOB", "RACE_WW", "RACE_RW", "RACE_XB", "MISMATCH", "BANK", "UNCOALESCED", "UNINIT", "LIMIT"]
@@ -64,7 +64,7 @@ class PgSummary(ctypes.Structure):
     _fields_ = [("instances", ctypes.c_uint64), ("n_fail", ctypes.c_uint64), ("n_records", ctypes.c_uint64),
                 ("first_key", ctypes.c_int64), ("first_launch", ctypes.c_uint32),
                 ("first_seed_idx", ctypes.c_uint32), ("per_kind", ctypes.c_uint64 * N_KINDS),
-                ("first_key_kind", ctypes.c_int64 * N_KINDS)]
+                ("first_key_kind", ctypes.c_int64 * N_KINDS), ("ir_ops", ctypes.c_uint64)]
 
 
 class PgError(RuntimeError):
@@ -76,7 +76,8 @@ class PgError(RuntimeError):
 _lib = None
 EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
            "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_seed_oblivious",
-           "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
+           "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals", "pg_measure_int32_peak",
+           "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
 
 
 def lib():
@@ -109,13 +110,17 @@ def lib():
     L.pg_ir_compile.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32]
     L.pg_run_timing.argtypes = [vp, ctypes.POINTER(ctypes.c_float), ctypes.POINTER(ctypes.c_float),
                                 ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint64)]
+    L.pg_run_intervals.argtypes = [vp, vp, ctypes.POINTER(ctypes.c_float), ctypes.c_size_t,
+                                   ctypes.POINTER(ctypes.c_size_t)]
+    L.pg_measure_int32_peak.argtypes = [vp, ctypes.POINTER(ctypes.c_double)]
     L.pg_last_error.restype = ctypes.c_char_p
     L.pg_version.restype = ctypes.c_char_p
     L.pg_ir_free.argtypes = [vp]
     L.pg_run_free.argtypes = [vp]
     for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
               "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info",
-              "pg_ir_seed_oblivious", "pg_ir_source", "pg_ir_compile", "pg_run_timing"):
+              "pg_ir_seed_oblivious", "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals",
+              "pg_measure_int32_peak"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -182,6 +187,21 @@ def _launch(l) -> PgLaunch:
     return o
 
 
+def _counter_ptr(t, n: int, what: str):
+    """Device pointer of a caller-owned counter tensor (pg_space.d_first_key / d_counts):
+    the library writes n int64 values through it, so it must be a contiguous int64 CUDA
+    tensor of >= n elements on the current device."""
+    if t is None:
+        return None
+    import torch
+    ok = (isinstance(t, torch.Tensor) and t.device.type == "cuda" and t.dtype == torch.int64
+          and t.is_contiguous() and t.numel() >= n and t.device.index == torch.cuda.current_device())
+    if not ok:
+        raise PgError(PG_E_ARG, "%s must be a contiguous int64 CUDA tensor of >= %d elements on the current "
+                                "device" % (what, n))
+    return t.data_ptr()
+
+
 @dataclass
 class Space:
     """Python side of pg_space.  Launches are Launch objects or (gdim, bdim, scalars)."""
@@ -216,8 +236,8 @@ class Space:
         sp.checks, sp.bank_model, sp.max_cex = self.checks, self.bank_model, self.max_cex
         sp.rank, sp.world = self.rank, self.world
         sp.cuda_stream = self.stream or None
-        sp.d_first_key = self.first_key.data_ptr() if self.first_key is not None else None
-        sp.d_counts = self.counts.data_ptr() if self.counts is not None else None
+        sp.d_first_key = _counter_ptr(self.first_key, 11, "first_key")
+        sp.d_counts = _counter_ptr(self.counts, 16, "counts")
         return sp, (ls, lt)
 
 
@@ -240,10 +260,10 @@ class Run:
                                  ctypes.byref(summ)))
         arr = buf[:min(n.value, cap, self.space.max_cex or (1 << 20))]   # the run keeps max_cex
         recs = arr.tolist() if tuples else arr
-        s = {"instances": summ.instances, "n_fail": summ.n_fail, "n_records": summ.n_records,
+        s = {"instances": summ.instances, "n_fail": summ.n_fail, "n_records": summ.n_records, "n_local": n.value,
              "first_key": summ.first_key, "first_launch": summ.first_launch,
              "first_seed_idx": summ.first_seed_idx, "per_kind": list(summ.per_kind),
-             "first_key_kind": list(summ.first_key_kind)}
+             "first_key_kind": list(summ.first_key_kind), "ir_ops": summ.ir_ops}
         return recs, s
 
     def site_stats(self, max_sites: int):
@@ -281,6 +301,17 @@ class Run:
         _ck(lib().pg_run_timing(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(n), ctypes.byref(h)))
         return {"ms_eval": a.value, "ms_total": b.value, "launches": n.value, "h2d_bytes": h.value}
 
+    def intervals(self, ref_event=None):
+        """[(start_ms, end_ms)] of every evaluation-kernel launch of the run, relative to
+        ref_event (a torch.cuda.Event recorded before the check) or to the run's first
+        enqueued operation (pg_run_intervals)."""
+        ref = ctypes.c_void_p(ref_event.cuda_event) if ref_event is not None else None
+        n = ctypes.c_size_t()
+        _ck(lib().pg_run_intervals(self._h, ref, None, 0, ctypes.byref(n)))
+        buf = (ctypes.c_float * max(2, 2 * n.value))()
+        _ck(lib().pg_run_intervals(self._h, ref, buf, n.value, ctypes.byref(n)))
+        return [(buf[2 * i], buf[2 * i + 1]) for i in range(n.value)]
+
     def __del__(self):
         if getattr(self, "_h", None) and self._h.value and _lib is not None:
             _lib.pg_run_free(self._h)
@@ -314,6 +345,14 @@ def pg_check_property(k: Ir, post: Ir, space: Space) -> Run:
 
 
 check_equiv, check_races, check_banks, check_property = pg_check_equiv, pg_check_races, pg_check_banks, pg_check_property
+
+
+def measure_int32_peak(stream: int = 0):
+    """Integer ops/s of the current device (pg_measure_int32_peak): alu pipe (LOP3),
+    fma pipe (IMAD), both pipes alternating."""
+    out = (ctypes.c_double * 3)()
+    _ck(lib().pg_measure_int32_peak(ctypes.c_void_p(stream or None), out))
+    return {"alu": out[0], "fma": out[1], "mixed": out[2]}
 
 
 def version() -> str:
