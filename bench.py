@@ -30,15 +30,15 @@ sys.path.insert(0, ROOT)
 METRIC = "VC instances checked/sec (n x tid x round x seed)"
 UNIT = "instances/s"
 SEEDS_PER_GPU = 64
-# SURVEY.md §8(d) algorithmic work per instance (thread x round) of a reduction round:
-# ~10 integer IR ops + 2 shared loads + 1 shared store = 13 ops.
-OPS_PER_INSTANCE = 13
-SM_COUNT = 148
-ALU_LANES_PER_SM_CLK = 64   # IADD3/LOP3 alu pipe: 4 SMSP x 16 lanes/clk (B300_MICROARCH: rt_SMSP = 2)
+# the bounded sample the oracle is timed on (cpu_baseline, --impl reference) and the GPU is
+# timed on beside it: the C2 pairs restricted to N <= 2^13, seeds 0..15
+SAMPLE_LOG_N = 13
+SAMPLE_SEEDS = 16
 
 
 WORKLOADS = {
-    # name: (description, seeds per GPU, ops per instance, builder(seeds))
+    # name: (description, seeds per GPU, (unused), builder(seeds)); the useful work per step is
+    # counted by the library itself (PG_CHK_OPCOUNT)
     "c2": ("C2: SDK reduce0 vs reduce1..6 + reduce2 vs reduce2_obo, B=2^0..2^10, N=B..2^16, "
            "%d RAND32 seeds per GPU, checks EQUIV|RACE|OOB", 64, 13, lambda W, s: W.c2(n_seeds=s)),
     "c1": ("C1: naive vs shared-memory transpose, bdim in [1,4]^2, up to 16x16 threads (1089 launches), "
@@ -146,17 +146,6 @@ def measured_peaks():
         return {}
 
 
-def ncu_profile():
-    """The committed ncu summary of the evaluation kernel for this workload ({} if none):
-    profiles/r1/k2_traffic.json for C2, profiles/r1/<workload>/k2_traffic.json otherwise."""
-    p = os.path.join(ROOT, "profiles", "r1", *(() if WL == "c2" else (WL,)), "k2_traffic.json")
-    try:
-        with open(p) as f:
-            return json.load(f)
-    except (OSError, ValueError):
-        return {}
-
-
 # ---------------------------------------------------------------- CPU oracle (reference arm / cpu_baseline)
 def _oracle_shard(args):
     rank, world, pts_max_log_n, n_seeds = args
@@ -171,9 +160,9 @@ def _oracle_shard(args):
     return inst
 
 
-def oracle_sample(max_log_n=14, n_seeds=0):
+def oracle_sample(max_log_n=SAMPLE_LOG_N, n_seeds=SAMPLE_SEEDS):
     """The oracle as it stands, one process per host core over seed shards, on the
-    C2 pairs restricted to N <= 2^max_log_n and n_seeds seeds (default: one seed per core)."""
+    C2 pairs restricted to N <= 2^max_log_n and seeds 0..n_seeds-1."""
     import multiprocessing as mp
     sys.path.insert(0, ROOT)
     import oracle
@@ -212,6 +201,28 @@ def run_reference(args):
 
 
 # ---------------------------------------------------------------- GPU arm
+def k2_busy(runs, ref_ev):
+    """(union, sum) in ms of the evaluation-kernel launch intervals of one step's runs,
+    relative to the step's start event (launches of a pair's two kernels and of concurrent
+    pairs overlap: the union is K2's busy time)."""
+    iv = []
+    for r in runs:
+        iv.extend(r.intervals(ref_ev))
+    tot = sum(b - a for a, b in iv)
+    iv.sort()
+    union, cur_a, cur_b = 0.0, None, None
+    for a, b in iv:
+        if cur_b is None or a > cur_b:
+            if cur_b is not None:
+                union += cur_b - cur_a
+            cur_a, cur_b = a, b
+        else:
+            cur_b = max(cur_b, b)
+    if cur_b is not None:
+        union += cur_b - cur_a
+    return union, tot
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -219,21 +230,19 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="pgvc", choices=["pgvc", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--ref-log-n", type=int, default=13, help="reference arm: C2 sample N <= 2^k per step")
-    ap.add_argument("--ref-seeds", type=int, default=0, help="0: one seed per host core")
+    ap.add_argument("--ref-log-n", type=int, default=SAMPLE_LOG_N, help="oracle sample: C2 with N <= 2^k")
+    ap.add_argument("--ref-seeds", type=int, default=SAMPLE_SEEDS, help="oracle sample: seeds 0..k-1")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + 1 step, no JSON (for ncu launch lists)")
     ap.add_argument("--diag", action="store_true", help="print per-step enqueue / device / per-check times")
     ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS),
                     help="c2 (headline, BASELINE configs[1]); others: the remaining configs for reference")
-    ap.add_argument("--streams", type=int, default=1,
-                    help="streams the independent pairs are spread over (0: one per pair; default 1: one stream, "
-                         "DESIGN.md §6 'Concurrent pairs')")
+    ap.add_argument("--streams", type=int, default=0,
+                    help="streams the independent pairs are spread over (default 0: one per pair; 1: one stream)")
     ap.add_argument("--seeds", type=int, default=0, help="seeds per GPU (default: the workload's)")
     args = ap.parse_args()
-    global WL, SEEDS_PER_GPU, OPS_PER_INSTANCE
+    global WL, SEEDS_PER_GPU
     WL = args.workload
     SEEDS_PER_GPU = args.seeds or WORKLOADS[WL][1]
-    OPS_PER_INSTANCE = WORKLOADS[WL][2]
     if args.impl == "reference":
         run_reference(args)
         return
@@ -243,12 +252,17 @@ def main():
     world, rank, local = dist_env()
     dev = local % max(1, torch.cuda.device_count())   # ranks > #GPUs share devices (tests only)
     torch.cuda.set_device(dev)
+    backend = None
     if world > 1:
         backend = os.environ.get("PGVC_DIST_BACKEND", "nccl")   # gloo: several ranks on one GPU (tests)
         if backend == "nccl":
+            os.environ.setdefault("NCCL_DEBUG", "INFO")          # communicator init lines (ranks / nranks)
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
             dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
         else:
             dist.init_process_group(backend)
+        print("[pgvc] rank %d/%d on cuda:%d, %s process group initialised" % (rank, world, dev, backend),
+              file=sys.stderr, flush=True)
     from paper_conf_ipps_lig12_b200 import build, distributed, pgvc
     if rank == 0 or world == 1:
         build.build()
@@ -256,14 +270,14 @@ def main():
         dist.barrier()
     wls = c2_pairs()
     irs = {}
+    from paper_conf_ipps_lig12_b200 import workloads as W
     for w in wls:
         for name in (w.src, w.tgt):
             if name not in irs:
-                from paper_conf_ipps_lig12_b200 import workloads as W
                 irs[name] = pgvc.load_ir(W.subject(name))
     stream = torch.cuda.Stream()
-    # the pairs are independent checks: with --streams S > 1 they are spread over S side
-    # streams forked from and joined back into `stream` (each pair has its own key/count rows)
+    # the pairs are independent checks: spread over S side streams forked from and joined
+    # back into `stream` (default: one per pair); each pair has its own key/count rows
     n_side = args.streams if args.streams > 0 else len(wls)
     side = [torch.cuda.Stream() for _ in range(n_side)] if n_side > 1 else [stream]
     pair_keys = torch.empty(len(wls), 11, dtype=torch.int64, device="cuda")
@@ -272,27 +286,34 @@ def main():
     step_counts = torch.zeros(16, dtype=torch.int64, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 
-    def step(keys_out, counts_out):
-        """One pass of the whole path over the workload (enqueue only): H1..H8 per pair, H9 at the end."""
+    def spaces(extra_checks=0, ns_fn=None):
+        out = []
+        for i, w in enumerate(wls):
+            # weak scaling: 64 seeds per GPU, seeds j = rank, rank + N, ... of a 64 x N seed space
+            ns = SEEDS_PER_GPU * world if w.input_mode != 1 else w.n_seeds   # exhaustive 0/1 sets are fixed
+            out.append(pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=ns, rank=rank, world=world,
+                                  input_mode=w.input_mode, input_range=w.input_range,
+                                  checks=w.checks | extra_checks, stream=side[i % len(side)].cuda_stream,
+                                  first_key=pair_keys[i], counts=pair_counts[i]))
+        return out
+    sps = spaces()
+
+    def step(keys_out, counts_out, sp_list=None):
+        """One pass of the whole path over the workload (enqueue only): H1..H8 per pair, the
+        pairs' counters merged on the device (K5), H9 across ranks at the end."""
         runs = []
         fork = torch.cuda.Event()
         fork.record(stream)
-        for i, w in enumerate(wls):
+        for i, (w, sp) in enumerate(zip(wls, sp_list or sps)):
             st = side[i % len(side)]
             if st is not stream and i < len(side):
                 st.wait_event(fork)
-            # weak scaling: 64 seeds per GPU, seeds j = rank, rank + N, ... of a 64 x N seed space
-            ns = SEEDS_PER_GPU * world if w.input_mode != 1 else w.n_seeds   # exhaustive 0/1 sets are fixed
-            sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=ns, rank=rank, world=world,
-                            input_mode=w.input_mode, input_range=w.input_range,
-                            checks=w.checks, stream=st.cuda_stream, first_key=pair_keys[i], counts=pair_counts[i])
             runs.append(pgvc.check_equiv(irs[w.src], irs[w.tgt], sp))
+        for st in side:
+            if st is not stream:
+                stream.wait_stream(st)
+        pgvc.merge_counters(pair_keys, pair_counts, keys_out, counts_out, stream.cuda_stream)
         with torch.cuda.stream(stream):
-            for st in side:
-                if st is not stream:
-                    stream.wait_stream(st)
-            torch.amin(pair_keys, 0, out=keys_out)
-            torch.sum(pair_counts, 0, out=counts_out)
             distributed.reduce_summary(keys_out, counts_out)   # H9: the only cross-GPU traffic
         return runs
 
@@ -303,8 +324,8 @@ def main():
             d2h += 64 * len(recs) + 8 * (16 + 11)
         return d2h
 
-    # warm-up (also JIT-compiles every evaluation kernel variant, builds the plans, and sizes the
-    # memory pool for K steps in flight, the pattern of the device-timed phase)
+    # warm-up (also JIT-compiles every evaluation kernel variant, builds the plans and their
+    # workspaces, captures the check graphs)
     collect(step(step_keys, step_counts))
     if not args.profile:
         for _ in range(max(1, args.warmup - 1)):
@@ -321,8 +342,17 @@ def main():
         torch.cuda.cudart().cudaProfilerStop()
         return
 
-    # ---- device-timed phase: K steps enqueued back to back (L2 flush between steps, outside the
-    # timed events); host hiccups are absorbed by the queued work
+    # ---- measurement-only passes (outside the timed region): the INT32 peak of this device,
+    # and the useful work of one step = the IR integer operations the subject kernels execute
+    # (PG_CHK_OPCOUNT: each instance once, no re-runs)
+    peak = pgvc.measure_int32_peak(stream.cuda_stream)
+    ops_runs = step(step_keys, step_counts, spaces(pgvc.CHK_OPCOUNT))
+    torch.cuda.synchronize()
+    ir_ops = sum(r.collect(cap=1)[1]["ir_ops"] for r in ops_runs)   # this rank's
+    del ops_runs
+
+    # ---- device-timed phase: K steps enqueued back to back (L2 flushed before every step,
+    # outside its events); each step replays the captured check graphs
     keys = [torch.empty(11, dtype=torch.int64, device="cuda") for _ in range(args.steps)]
     cnts = [torch.empty(16, dtype=torch.int64, device="cuda") for _ in range(args.steps)]
     clocks = Clocks(dev)
@@ -332,16 +362,14 @@ def main():
     torch.cuda.synchronize()
     clocks.start()
     clocks.wait_first()
-    evs, all_runs, host_ms = [], [], []
+    evs, all_runs = [], []
     for k in range(args.steps):
         with torch.cuda.stream(stream):
             flush.fill_(1)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        h0 = time.perf_counter()
         e0.record(stream)
         all_runs.append(step(keys[k], cnts[k]))
         e1.record(stream)
-        host_ms.append(1000 * (time.perf_counter() - h0))
         evs.append((e0, e1))
     clocks.wait_sample(timeout=2.0)   # (the enqueued steps are still running: a sample under load)
     torch.cuda.synchronize()
@@ -352,76 +380,109 @@ def main():
     step_ms = [e0.elapsed_time(e1) for e0, e1 in evs]
     dev_ms = sum(step_ms)
     inst_total = sum(int(c[0].item()) for c in cnts)      # whole job: counts are all-reduced over ranks
-    launches, h2d, eval_ms = 0, 0, 0.0
-    for runs in all_runs:
+    launches, h2d, k2_union, k2_sum = 0, 0, [], []
+    for (e0, _), runs in zip(evs, all_runs):
+        u, t = k2_busy(runs, e0)
+        k2_union.append(u)
+        k2_sum.append(t)
         for r in runs:
-            t = r.timing()
-            launches += t["launches"]
-            h2d += t["h2d_bytes"]
-            eval_ms += t["ms_eval"]
+            tm = r.timing()
+            launches += tm["launches"]
+            h2d += tm["h2d_bytes"]
     if args.diag and rank == 0:
-        print("device ms per step:", ["%.1f" % x for x in step_ms], file=sys.stderr)
-        print("host enqueue ms per step:", ["%.1f" % x for x in host_ms], file=sys.stderr)
+        print("device ms per step:", ["%.2f" % x for x in step_ms], file=sys.stderr)
+        print("K2 busy (union) ms per step:", ["%.2f" % x for x in k2_union], file=sys.stderr)
         print("step keys/counts:", keys[-1].tolist(), cnts[-1].tolist(), file=sys.stderr)
     del all_runs
 
-    # ---- end-to-end phase: the same steps through the C ABI, host launch lists in, records and
-    # counters read back every step (wall clock)
-    wall_s, d2h = 0.0, 0
+    # ---- end-to-end phase: the same steps through the C ABI from an idle device, host launch
+    # lists in, records and counters read back every step (wall clock); the enqueue part of
+    # each step is the host cost of the path
+    wall_s, d2h, enq_ms = 0.0, 0, []
     for k in range(args.steps):
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         runs = step(keys[k], cnts[k])
+        enq_ms.append(1000 * (time.perf_counter() - t0))
         d2h += collect(runs)
         torch.cuda.synchronize()
         wall_s += time.perf_counter() - t0
         del runs
-    t = torch.tensor([dev_ms, wall_s], dtype=torch.float64, device="cuda")
+    t = torch.tensor([dev_ms, wall_s, sum(k2_union)], dtype=torch.float64, device="cuda")
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    dev_ms, wall_s = float(t[0]), float(t[1])
+    dev_ms, wall_s, k2_ms = float(t[0]), float(t[1]), float(t[2])
     value = inst_total / (dev_ms / 1000.0)
     e2e = inst_total / wall_s
-    peaks = measured_peaks()
-    sm_max = clk.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
-    alu_peak = SM_COUNT * ALU_LANES_PER_SM_CLK * sm_max * 1e6
-    per_gpu_inst = inst_total / world
-    # K2 time: with one stream, the sum of the evaluation launches' durations (CUDA events around
-    # each); with the pairs on concurrent streams those launches overlap each other and the other
-    # kernels, so a launch's duration is no longer the kernel's own - the whole device step time is
-    # used instead (a lower bound on K2's achieved rate: it also covers K1/K2b/K3/K4)
-    k2_basis = "k2_launches" if len(side) == 1 else "whole_step"
-    k2_s = eval_ms / 1000.0 if len(side) == 1 else dev_ms / 1000.0
-    achieved_ops = per_gpu_inst * OPS_PER_INSTANCE / k2_s if k2_s else None
+    sm_max = clk.get("sm_max_mhz") or measured_peaks().get("sm_max_mhz", 1965.0)
+    # roofline (per GPU): useful IR integer ops of this rank's step / K2 busy time, against
+    # the measured integer peak of both pipes (alu: IADD3/LOP3/SHF/ISETP, fma: IMAD)
+    k2_s = k2_ms / 1000.0 / args.steps
+    achieved = ir_ops / k2_s if k2_s else None
+    per_gpu_inst = inst_total / world / args.steps
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": workload_desc(), "seeds_per_gpu": SEEDS_PER_GPU, "l2": "flushed between steps",
-                   "streams": len(side),
-                   "parallelism": "dp%d over seeds" % world},
-        "roofline": {"bound": "alu", "achieved": achieved_ops / 1e12 if achieved_ops else None,
-                     "peak": alu_peak / 1e12, "unit": "Tops/s (int32, algorithmic IR ops)",
-                     "frac": (achieved_ops / alu_peak) if achieved_ops else None,
-                     "traffic": ncu_profile().get("bytes_per_launch"),
-                     "ncu_issue_active_pct": ncu_profile().get("issue_active_pct_time_weighted"),
-                     "kernel": "pgk_eval (K2)", "ops_per_instance": OPS_PER_INSTANCE,
-                     "k2_ms_per_step": eval_ms / args.steps, "time_basis": k2_basis, "streams": len(side),
-                     "peak_source": "148 SM x 64 int32 lanes/clk x sm_max_mhz (DESIGN.md §6)"},
+        "config": {"workload": workload_desc(), "seeds_per_gpu": SEEDS_PER_GPU, "l2": "flushed before every step",
+                   "streams": len(side), "parallelism": "dp%d over seeds" % world},
+        "roofline": {"bound": "alu", "achieved": achieved / 1e12 if achieved else None,
+                     "peak": peak["mixed"] / 1e12, "unit": "Tops/s (int32 IR operations)",
+                     "frac": (achieved / peak["mixed"]) if achieved else None, "traffic": None,
+                     "kernel": "pgk_eval (K2)", "ir_ops_per_step": ir_ops,
+                     "ir_ops_per_instance": ir_ops / per_gpu_inst if per_gpu_inst else None,
+                     "k2_busy_ms_per_step": k2_ms / args.steps,
+                     "k2_launch_sum_ms_per_step": sum(k2_sum) / args.steps,
+                     "k2_share_of_step": k2_ms / dev_ms if dev_ms else None,
+                     "peak_source": "measured live: pg_measure_int32_peak, LOP3 + IMAD chains on both pipes",
+                     "peak_alu_pipe": peak["alu"] / 1e12, "peak_fma_pipe": peak["fma"] / 1e12,
+                     "frac_of_alu_pipe": (achieved / peak["alu"]) if achieved else None,
+                     "time_basis": "union of K2 launch intervals (CUDA events in the check graphs)"},
         "e2e": {"value": e2e, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
                 "d2h_bytes_per_step": d2h // args.steps},
         "step_ms": {"median": statistics.median(step_ms), "min": min(step_ms), "max": max(step_ms),
-                    "host_enqueue_median": statistics.median(host_ms)},
+                    "host_enqueue_median": statistics.median(enq_ms)},
         "gpu_launches": launches // args.steps * args.steps,
         "clocks": clk,
+        # the last timed step's H9-reduced summary (whole job): first failing key, counts
+        "check": {"first_key": int(keys[-1][0].item()), "instances": int(cnts[-1][0].item()),
+                  "n_fail": int(cnts[-1][12].item()), "records": int(cnts[-1][11].item()),
+                  "per_kind": [int(x) for x in cnts[-1][1:11].tolist()]},
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        inst, dt, cores, sample = oracle_sample()
+        # like for like: the oracle and the GPU on the same bounded sample (C2 with N <= 2^k, seeds
+        # 0..S-1), then the oracle's number as the CPU baseline
+        inst, dt, cores, sample = oracle_sample(max_log_n=args.ref_log_n, n_seeds=args.ref_seeds)
         line["cpu_baseline"] = {"value": inst / dt, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
+        g_inst, g_s = gpu_sample(pgvc, irs, stream, args.ref_log_n, args.ref_seeds)
+        line["same_sample"] = {"sample": sample, "oracle": inst / dt, "gpu": g_inst / g_s,
+                               "instances_match": g_inst == inst}
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def gpu_sample(pgvc, irs, stream, max_log_n, n_seeds, reps=5):
+    """The GPU on the oracle's sample (same pairs, launches and seeds; best of reps, device time)."""
+    import torch
+    from paper_conf_ipps_lig12_b200 import workloads as W
+    wls = W.c2(n_seeds=n_seeds, max_log_n=max_log_n, max_log_b=10)
+    fk = torch.empty(len(wls), 11, dtype=torch.int64, device="cuda")
+    ct = torch.empty(len(wls), 16, dtype=torch.int64, device="cuda")
+    sps = [pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=n_seeds, checks=w.checks, stream=stream.cuda_stream,
+                      first_key=fk[i], counts=ct[i]) for i, w in enumerate(wls)]
+    best, inst = None, 0
+    for _ in range(reps + 1):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        runs = [pgvc.check_equiv(irs[w.src], irs[w.tgt], sp) for w, sp in zip(wls, sps)]
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1)
+        inst = sum(r.collect(cap=1)[1]["instances"] for r in runs)
+        best = ms if best is None else min(best, ms)
+    return inst, best / 1000.0
 
 
 if __name__ == "__main__":

@@ -209,6 +209,13 @@ int pg_run_timing(pg_run *r, float *ms_eval, float *ms_total, uint32_t *n_launch
  * are written.  Synchronises the run's stream. */
 int pg_run_intervals(pg_run *r, void *ref_event, float *buf, size_t cap, size_t *n);
 
+/* Merge the counters of n_rows checks enqueued on the same device (e.g. the pairs of one
+ * step, each with its own rows): d_out_first_key[i] = MIN over rows of d_first_keys[r*11+i],
+ * d_out_counts[i] = SUM over rows of d_counts[r*16+i] - the reduction H9 then applies across
+ * ranks.  All pointers are device int64 buffers (borrowed); enqueued on `stream`. */
+int pg_merge_counters(const int64_t *d_first_keys, const int64_t *d_counts, uint32_t n_rows,
+                      int64_t *d_out_first_key, int64_t *d_out_counts, void *stream);
+
 /* Measurement utility (not part of the method; the K2 roofline denominator, SURVEY.md
  * §8(d)): integer ops/s the current device sustains on `stream` for [0] LOP3 chains (alu
  * pipe), [1] IMAD chains (fma pipe), [2] both alternating (the two pipes together).

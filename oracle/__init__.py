@@ -235,3 +235,44 @@ def sm64(x: int) -> int:
 
 def rand32(seed: int, tag: int, idx: int) -> int:
     return lib().or_rand32(seed, tag, idx)
+
+
+def _check_shard(args):
+    src, tgt, launch_src, launch_tgt, kw, rank, world = args
+    return check(src, tgt, launch_src, launch_tgt, rank=rank, world=world, **kw)
+
+
+def check_parallel(src: str, tgt, launch_src, launch_tgt=None, *, processes=0, **kw):
+    """check() over host cores: one process per seed shard (the oracle's own rank/world
+    sharding, seed j -> shard j mod world), results merged as H9 merges ranks - counts
+    summed, first keys MIN, records (one per slot, so unique keys) in key order.  Test
+    infrastructure, like check()."""
+    import multiprocessing as mp
+    n_seeds = kw.get("n_seeds", 1)
+    world = max(1, min(processes or len(os.sched_getaffinity(0)), n_seeds))
+    if kw.get("world", 1) != 1 or kw.get("rank", 0) != 0:
+        raise ValueError("check_parallel shards by itself")
+    kw = {k: v for k, v in kw.items() if k not in ("rank", "world")}
+    build()
+    if world == 1:
+        return check(src, tgt, launch_src, launch_tgt, **kw)
+    launch_src = [tuple(map(tuple, (l.gdim, l.bdim, l.scalars))) if hasattr(l, "gdim") else l for l in launch_src]
+    if launch_tgt is not None:
+        launch_tgt = [tuple(map(tuple, (l.gdim, l.bdim, l.scalars))) if hasattr(l, "gdim") else l
+                      for l in launch_tgt]
+    with mp.get_context("fork").Pool(world) as pool:
+        parts = pool.map(_check_shard, [(src, tgt, launch_src, launch_tgt, kw, r, world) for r in range(world)])
+    recs = sorted((r for p in parts for r in p["records"]), key=lambda r: r[0])
+    counts = [sum(p["counts"][i] for p in parts) for i in range(16)]
+    first = [min(p["first_key"][i] for p in parts) for i in range(11)]
+    stats = None
+    if parts[0]["site_stats"] is not None:
+        stats = parts[0]["site_stats"].copy()
+        for p in parts[1:]:
+            s = p["site_stats"]
+            stats[..., 0] = np.maximum(stats[..., 0], s[..., 0])
+            stats[..., 3] = np.maximum(stats[..., 3], s[..., 3])
+            for c in (1, 2, 4, 5, 6, 7):
+                stats[..., c] += s[..., c]
+    return {"records": recs, "n_records": sum(p["n_records"] for p in parts), "counts": counts,
+            "first_key": first, "site_stats": stats}

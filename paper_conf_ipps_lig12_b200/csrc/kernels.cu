@@ -313,6 +313,23 @@ __global__ void pg_reset_counters(long long* first_key, long long* counts) {
     if (i < 16) counts[i] = 0;
 }
 
+// K5: merge the counters of several checks (rows of first keys int64[11] and counts
+// int64[16]): MIN of the keys, SUM of the counts - the same reduction H9 applies across ranks.
+__global__ void pg_merge_counters(const long long* keys, const long long* counts, u32 n, long long* out_keys,
+                                  long long* out_counts) {
+    const u32 i = threadIdx.x;
+    if (i < 11) {
+        long long m = 0x7FFFFFFFFFFFFFFFll;
+        for (u32 r = 0; r < n; r++) m = min(m, keys[(u64)r * 11u + i]);
+        out_keys[i] = m;
+    }
+    if (i < 16) {
+        long long s = 0;
+        for (u32 r = 0; r < n; r++) s += counts[(u64)r * 16u + i];
+        out_counts[i] = s;
+    }
+}
+
 __device__ __forceinline__ bool kind_failing(u32 kind, u32 banks_mode) {
     return kind <= PGK_MISMATCH || kind == PGK_LIMIT || (banks_mode && (kind == PGK_BANK || kind == PGK_UNCOAL));
 }
@@ -457,6 +474,12 @@ __global__ void __launch_bounds__(1024) pg_count_reduce(const u64* inst_cnt, u32
     }
 }
 
+// Condition of a captured re-run block (a conditional IF node of the check graph): run the
+// block only if some instance of the batch was flagged.
+__global__ void pg_set_cond(cudaGraphConditionalHandle h, const u32* flag) {
+    cudaGraphSetConditional(h, *(volatile const u32*)flag != 0u ? 1u : 0u);
+}
+
 // ------------------------------------------------------------------ INT32 peak microbenchmark
 // Measurement only (the roofline denominator of K2): 8 independent
 // chains per thread of LOP3 (alu pipe, mode 0), IMAD (fma pipe, mode 1) or both
@@ -491,15 +514,27 @@ __global__ void __launch_bounds__(256) pg_int_peak(u32 iters, u32* sink) {
 // ------------------------------------------------------------------ host wrappers (C++ linkage, used by api.cpp)
 namespace pgk {
 
-// grid.x of the per-(job, instance) kernels: enough CTAs for a CTA per instance, capped
-// (re-initialisation of flagged instances: a few CTAs per job walk its instances)
+// SMs of the current device (queried once per device): grids of the CTA-task kernels stride
+// over their tasks with <= 16 CTAs per SM
+u32 sm_count() {
+    static int cache[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148u;
+    if (!cache[dev]) {
+        int n = 0;
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        cache[dev] = n > 0 ? n : 148;
+    }
+    return (u32)cache[dev];
+}
+u32 task_grid(u32 n_tasks) { return n_tasks < sm_count() * 16u ? n_tasks : sm_count() * 16u; }
 
 
 cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 task_base, u32 n_tasks, u32* arena_s, u32* arena_t,
                        u32* input, u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags,
                        const u32* any) {
     if (!n_jobs || !n_tasks) return cudaSuccess;
-    const u32 grid = n_tasks < 148u * 16u ? n_tasks : 148u * 16u;
+    const u32 grid = task_grid(n_tasks);
     pg_gen_inputs<<<grid, 256, 0, st>>>(jobs, n_jobs, task_base, n_tasks, arena_s, arena_t, input, seed_base, mode,
                                         range, mask, flags, any);
     return cudaGetLastError();
@@ -521,7 +556,7 @@ cudaError_t count_reduce(const u64* inst_cnt, u32 n, long long* counts, cudaStre
 cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 n_tasks, u32 max_inst, const u32* arena_s,
                     const u32* arena_t, const u32* input, PgSlot* slots, u64* mm_key, cudaStream_t st) {
     if (!n_jobs) return cudaSuccess;
-    pg_compare<<<n_tasks < 148u * 16u ? n_tasks : 148u * 16u, 256, 0, st>>>(jobs, n_jobs, n_tasks, arena_s, arena_t,
+    pg_compare<<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, arena_s, arena_t,
                                                                             input, slots, mm_key);
     for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
         const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
@@ -546,7 +581,7 @@ cudaError_t lockstep(const PgLock* jobs, u32 n_jobs, u32 max_inst, const u32* ar
 cudaError_t xb_detect(const PgXb* jobs, u32 n_jobs, u32 n_tasks, const u32* arena, u32* flags, u32* any,
                       cudaStream_t st) {
     if (!n_jobs || !n_tasks) return cudaSuccess;
-    pg_xb_detect<<<n_tasks < 148u * 16u ? n_tasks : 148u * 16u, 256, 0, st>>>(jobs, n_jobs, n_tasks, arena, flags,
+    pg_xb_detect<<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, arena, flags,
                                                                               any);
     return cudaGetLastError();
 }
@@ -561,6 +596,12 @@ cudaError_t stats_reduce(const PgWork* items, u32 n_items, const u64* item_stats
                          u32 max_sites, cudaStream_t st) {
     if (!n_items) return cudaSuccess;
     pg_stats_reduce<<<n_items, 128, 0, st>>>(items, item_stats, flags, launch_stats, max_sites);
+    return cudaGetLastError();
+}
+
+cudaError_t merge_counters(const long long* keys, const long long* counts, u32 n, long long* out_keys,
+                           long long* out_counts, cudaStream_t st) {
+    pg_merge_counters<<<1, 32, 0, st>>>(keys, counts, n, out_keys, out_counts);
     return cudaGetLastError();
 }
 
@@ -583,6 +624,11 @@ cudaError_t compact(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 
     if (!n_inst) return cudaSuccess;
     pg_compact<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, inst_nrec, offsets,
                                                      (PgCexDev*)out, cap, total);
+    return cudaGetLastError();
+}
+
+cudaError_t set_cond(cudaGraphConditionalHandle h, const u32* flag, cudaStream_t st) {
+    pg_set_cond<<<1, 1, 0, st>>>(h, flag);
     return cudaGetLastError();
 }
 

@@ -76,7 +76,8 @@ class PgError(RuntimeError):
 _lib = None
 EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
            "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_seed_oblivious",
-           "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals", "pg_measure_int32_peak",
+           "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals", "pg_merge_counters",
+           "pg_measure_int32_peak",
            "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
 
 
@@ -113,6 +114,7 @@ def lib():
     L.pg_run_intervals.argtypes = [vp, vp, ctypes.POINTER(ctypes.c_float), ctypes.c_size_t,
                                    ctypes.POINTER(ctypes.c_size_t)]
     L.pg_measure_int32_peak.argtypes = [vp, ctypes.POINTER(ctypes.c_double)]
+    L.pg_merge_counters.argtypes = [vp, vp, ctypes.c_uint32, vp, vp, vp]
     L.pg_last_error.restype = ctypes.c_char_p
     L.pg_version.restype = ctypes.c_char_p
     L.pg_ir_free.argtypes = [vp]
@@ -120,7 +122,7 @@ def lib():
     for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
               "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info",
               "pg_ir_seed_oblivious", "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals",
-              "pg_measure_int32_peak"):
+              "pg_merge_counters", "pg_measure_int32_peak"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -222,10 +224,18 @@ class Space:
     counts: object = None           # torch int64[16] on the device (optional)
 
     def marshal(self):
-        ls = (PgLaunch * max(1, len(self.launch_src)))(*[_launch(l) for l in self.launch_src])
-        lt = None
-        if self.launch_tgt is not None:
-            lt = (PgLaunch * max(1, len(self.launch_tgt)))(*[_launch(l) for l in self.launch_tgt])
+        # (the launch arrays are built once per Space object: a Space re-used for every step
+        # of a loop marshals its launch lists once)
+        key = (id(self.launch_src), len(self.launch_src), id(self.launch_tgt))
+        cached = self.__dict__.get("_launch_arrays")
+        if cached is not None and cached[0] == key:
+            ls, lt = cached[1], cached[2]
+        else:
+            ls = (PgLaunch * max(1, len(self.launch_src)))(*[_launch(l) for l in self.launch_src])
+            lt = None
+            if self.launch_tgt is not None:
+                lt = (PgLaunch * max(1, len(self.launch_tgt)))(*[_launch(l) for l in self.launch_tgt])
+            self.__dict__["_launch_arrays"] = (key, ls, lt)
         sp = PgSpace()
         sp.launch_src = ctypes.cast(ls, ctypes.POINTER(PgLaunch))
         sp.launch_tgt = ctypes.cast(lt, ctypes.POINTER(PgLaunch)) if lt is not None else None
@@ -345,6 +355,19 @@ def pg_check_property(k: Ir, post: Ir, space: Space) -> Run:
 
 
 check_equiv, check_races, check_banks, check_property = pg_check_equiv, pg_check_races, pg_check_banks, pg_check_property
+
+
+def merge_counters(first_keys, counts, out_first_key, out_counts, stream: int = 0):
+    """pg_merge_counters: MIN over the rows of first_keys (n x 11), SUM over the rows of counts
+    (n x 16), into out_first_key (11) / out_counts (16); int64 CUDA tensors."""
+    n = first_keys.shape[0]
+    if counts.shape[0] != n or first_keys.shape[1:] != (11,) or counts.shape[1:] != (16,):
+        raise PgError(PG_E_ARG, "first_keys must be (n, 11) and counts (n, 16)")
+    _ck(lib().pg_merge_counters(ctypes.c_void_p(_counter_ptr(first_keys, 11 * n, "first_keys")),
+                                ctypes.c_void_p(_counter_ptr(counts, 16 * n, "counts")), n,
+                                ctypes.c_void_p(_counter_ptr(out_first_key, 11, "out_first_key")),
+                                ctypes.c_void_p(_counter_ptr(out_counts, 16, "out_counts")),
+                                ctypes.c_void_p(stream or None)))
 
 
 def measure_int32_peak(stream: int = 0):

@@ -70,3 +70,13 @@ def test_fake_world_shards_union(oracle, W):
         assert D.merge_records([p["records"] for p in parts]) == full["records"]
         assert min(p["first_key"][0] for p in parts) == full["first_key"][0]
         assert [sum(p["counts"][i] for p in parts) for i in range(16)] == full["counts"]
+
+
+def test_oracle_check_parallel_equals_serial(oracle, W):
+    # the host-parallel oracle (seed shards over processes, merged as H9 merges ranks) used
+    # by the full-size GPU parity tests gives exactly the serial oracle's result
+    w = W.c2_pair("reduce2", "reduce2_obo", n_seeds=5, max_log_n=7, max_log_b=5)
+    args = (W.subject(w.src), W.subject(w.tgt), w.launch_src, w.launch_tgt)
+    a = oracle.check(*args, n_seeds=5, checks=w.checks, cap=1 << 20)
+    b = oracle.check_parallel(*args, n_seeds=5, checks=w.checks, cap=1 << 20, processes=3)
+    assert a["records"] == b["records"] and a["counts"] == b["counts"] and a["first_key"] == b["first_key"]

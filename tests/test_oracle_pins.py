@@ -234,3 +234,26 @@ def test_ww_record_is_the_committed_write_and_the_writer_pair(oracle):
         (0, 0x100, 0, 0, 3, 0, 10, 0)
     _, fin, _ = oracle.exec_kernel(WW, one(bdim=(4, 1, 1)), 0)
     assert [int(x) for x in fin[0]] == [10 + 22] * 4   # s[1] committed by thread 2 (min writer)
+
+
+# ------------------------------------------------------------------ X19 loop fuel
+def test_loop_fuel_limit_record(oracle):
+    # X19: at most 2^20 loop back-edges per thread per round; the thread that exceeds it stops
+    # (exits) with a LIMIT record (round, no array, addr 0, its gtid, no second thread, no
+    # site, val_a = 2 marks the fuel limit; 1 marks the write-log limit)
+    k = """
+    kernel spin(global out int o[4]) {
+      int x = 0;
+      if (tid.x >= 1) { while (x >= 0) { x = x + 1; x = x & 0xFFFF; } }
+      o[tid.x] = 1;
+    }
+    """
+    r = oracle.check(k, None, [one(bdim=(3, 1, 1))], mode=oracle.MODE_RACES, checks=oracle.RACE | oracle.OOB)
+    (rec,) = r["records"]
+    d = dict(zip(oracle.REC_FIELDS, rec))
+    assert (d["kind"], d["round"], d["array"], d["addr"], d["tid_a"], d["tid_b"], d["site"], d["val_a"]) == \
+        (9, 0, 0xFFFFFFFF, 0, 1, 0xFFFFFFFF, 0xFFFFFFFF, 2)
+    assert d["count"] == 2                           # threads 1 and 2
+    _, fin, counts = oracle.exec_kernel(k, one(bdim=(3, 1, 1)), 0)
+    assert int(fin[0][0]) == 1                       # thread 0 finished; 1 and 2 never reached the store
+    assert counts[0] == 3
