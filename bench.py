@@ -41,6 +41,9 @@ WORKLOADS = {
     # counted by the library itself (PG_CHK_OPCOUNT)
     "c2": ("C2: SDK reduce0 vs reduce1..6 + reduce2 vs reduce2_obo, B=2^0..2^10, N=B..2^16, "
            "%d RAND32 seeds per GPU, checks EQUIV|RACE|OOB", 64, 13, lambda W, s: W.c2(n_seeds=s)),
+    "c2n": ("C2, the survey's design: reduce0..reduce6 and reduce2_obo each evaluated once per (N, B, seed), all 28 "
+            "pairs compared (pg_check_equiv_n; B = 1 points as a 4-kernel check), B=2^0..2^10, N=B..2^16, "
+            "%d RAND32 seeds per GPU, checks EQUIV|RACE|OOB", 64, None, lambda W, s: W.c2_all(n_seeds=s)),
     "c1": ("C1: naive vs shared-memory transpose, bdim in [1,4]^2, up to 16x16 threads (1089 launches), "
            "%d RAND32 seeds per GPU, checks EQUIV|RACE|OOB", 64, 14, lambda W, s: [W.c1(n_seeds=s)]),
     "c3": ("C3: Blelloch scan vs padded scan (LOG_NUM_BANKS 4 and 5) and the dropped-barrier mutant, n <= 2^14, "
@@ -147,15 +150,29 @@ def measured_peaks():
 
 
 # ---------------------------------------------------------------- CPU oracle (reference arm / cpu_baseline)
+def sample_workloads(max_log_n, n_seeds):
+    """The bounded sample of the headline workload (C2 restricted to N <= 2^max_log_n)."""
+    from paper_conf_ipps_lig12_b200 import workloads as W
+    if WL == "c2n":
+        return W.c2_all(n_seeds=n_seeds, max_log_n=max_log_n, max_log_b=10)
+    return W.c2(n_seeds=n_seeds, max_log_n=max_log_n, max_log_b=10)
+
+
 def _oracle_shard(args):
-    rank, world, pts_max_log_n, n_seeds = args
+    rank, world, pts_max_log_n, n_seeds, wl = args
+    global WL
+    WL = wl
     sys.path.insert(0, ROOT)
     import oracle
     from paper_conf_ipps_lig12_b200 import workloads as W
     inst = 0
-    for w in W.c2(n_seeds=n_seeds, max_log_n=pts_max_log_n, max_log_b=10):
-        r = oracle.check(W.subject(w.src), W.subject(w.tgt), w.launch_src, w.launch_tgt, n_seeds=n_seeds,
-                         rank=rank, world=world, checks=w.checks, cap=1 << 16)
+    for w in sample_workloads(pts_max_log_n, n_seeds):
+        if hasattr(w, "kernels"):
+            r = oracle.check_n([W.subject(n) for n in w.kernels], w.launches, n_seeds=n_seeds, rank=rank,
+                               world=world, checks=w.checks, cap=1 << 16)
+        else:
+            r = oracle.check(W.subject(w.src), W.subject(w.tgt), w.launch_src, w.launch_tgt, n_seeds=n_seeds,
+                             rank=rank, world=world, checks=w.checks, cap=1 << 16)
         inst += r["counts"][0]
     return inst
 
@@ -172,10 +189,10 @@ def oracle_sample(max_log_n=SAMPLE_LOG_N, n_seeds=SAMPLE_SEEDS):
     world = min(cores, n_seeds)
     t0 = time.perf_counter()
     with mp.get_context("fork").Pool(world) as pool:
-        inst = sum(pool.map(_oracle_shard, [(r, world, max_log_n, n_seeds) for r in range(world)]))
+        inst = sum(pool.map(_oracle_shard, [(r, world, max_log_n, n_seeds, WL) for r in range(world)]))
     dt = time.perf_counter() - t0
-    sample = ("C2 pairs restricted to N <= 2^%d (B = 2^0..2^10), seeds 0..%d, %d processes"
-              % (max_log_n, n_seeds - 1, world))
+    sample = ("%s restricted to N <= 2^%d (B = 2^0..2^10), seeds 0..%d, %d processes"
+              % ("C2 (all kernels once, all pairs)" if WL == "c2n" else "C2 pairs", max_log_n, n_seeds - 1, world))
     return inst, dt, world, sample
 
 
@@ -201,6 +218,17 @@ def run_reference(args):
 
 
 # ---------------------------------------------------------------- GPU arm
+def kernel_names(w):
+    return list(w.kernels) if hasattr(w, "kernels") else [w.src, w.tgt]
+
+
+def run_one(pgvc, irs, w, sp):
+    """One check of the workload: a pair (pg_check_equiv) or an N-kernel check."""
+    if hasattr(w, "kernels"):
+        return pgvc.check_equiv_n([irs[n] for n in w.kernels], w.launches, sp)
+    return pgvc.check_equiv(irs[w.src], irs[w.tgt], sp)
+
+
 def k2_busy(runs, ref_ev):
     """(union, sum) in ms of the evaluation-kernel launch intervals of one step's runs,
     relative to the step's start event (launches of a pair's two kernels and of concurrent
@@ -272,7 +300,7 @@ def main():
     irs = {}
     from paper_conf_ipps_lig12_b200 import workloads as W
     for w in wls:
-        for name in (w.src, w.tgt):
+        for name in kernel_names(w):
             if name not in irs:
                 irs[name] = pgvc.load_ir(W.subject(name))
     stream = torch.cuda.Stream()
@@ -290,9 +318,11 @@ def main():
         out = []
         for i, w in enumerate(wls):
             # weak scaling: 64 seeds per GPU, seeds j = rank, rank + N, ... of a 64 x N seed space
-            ns = SEEDS_PER_GPU * world if w.input_mode != 1 else w.n_seeds   # exhaustive 0/1 sets are fixed
-            out.append(pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=ns, rank=rank, world=world,
-                                  input_mode=w.input_mode, input_range=w.input_range,
+            mode = getattr(w, "input_mode", 0)
+            ns = SEEDS_PER_GPU * world if mode != 1 else w.n_seeds   # exhaustive 0/1 sets are fixed
+            ls, lt = (w.launches[0], None) if hasattr(w, "kernels") else (w.launch_src, w.launch_tgt)
+            out.append(pgvc.Space(ls, lt, n_seeds=ns, rank=rank, world=world,
+                                  input_mode=mode, input_range=getattr(w, "input_range", 0),
                                   checks=w.checks | extra_checks, stream=side[i % len(side)].cuda_stream,
                                   first_key=pair_keys[i], counts=pair_counts[i]))
         return out
@@ -308,7 +338,7 @@ def main():
             st = side[i % len(side)]
             if st is not stream and i < len(side):
                 st.wait_event(fork)
-            runs.append(pgvc.check_equiv(irs[w.src], irs[w.tgt], sp))
+            runs.append(run_one(pgvc, irs, w, sp))
         for st in side:
             if st is not stream:
                 stream.wait_stream(st)
@@ -466,17 +496,17 @@ def main():
 def gpu_sample(pgvc, irs, stream, max_log_n, n_seeds, reps=5):
     """The GPU on the oracle's sample (same pairs, launches and seeds; best of reps, device time)."""
     import torch
-    from paper_conf_ipps_lig12_b200 import workloads as W
-    wls = W.c2(n_seeds=n_seeds, max_log_n=max_log_n, max_log_b=10)
+    wls = sample_workloads(max_log_n, n_seeds)
     fk = torch.empty(len(wls), 11, dtype=torch.int64, device="cuda")
     ct = torch.empty(len(wls), 16, dtype=torch.int64, device="cuda")
-    sps = [pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=n_seeds, checks=w.checks, stream=stream.cuda_stream,
-                      first_key=fk[i], counts=ct[i]) for i, w in enumerate(wls)]
+    sps = [pgvc.Space(w.launches[0] if hasattr(w, "kernels") else w.launch_src,
+                      None if hasattr(w, "kernels") else w.launch_tgt, n_seeds=n_seeds, checks=w.checks,
+                      stream=stream.cuda_stream, first_key=fk[i], counts=ct[i]) for i, w in enumerate(wls)]
     best, inst = None, 0
     for _ in range(reps + 1):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        runs = [pgvc.check_equiv(irs[w.src], irs[w.tgt], sp) for w, sp in zip(wls, sps)]
+        runs = [run_one(pgvc, irs, w, sp) for w, sp in zip(wls, sps)]
         e1.record(stream)
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1)

@@ -80,7 +80,7 @@ typedef struct {
     const pg_launch *launch_src, *launch_tgt;  /* launch_tgt may be NULL (= launch_src) */
     uint32_t n_launch;                         /* < 2^18 */
     uint64_t seed_base;
-    uint32_t n_seeds;                          /* < 2^24 */
+    uint32_t n_seeds;                          /* < 2^21 */
     uint32_t input_mode, input_range;          /* PG_IN_*, k for PG_IN_RANGE */
     uint32_t bits;                             /* arithmetic width w (X2): 1..32, default 32 */
     uint32_t checks, bank_model, max_cex;      /* PG_CHK_* mask; PG_BANKS_*; max records kept */
@@ -94,7 +94,8 @@ typedef struct {
 
 /* One counterexample record (X16): the minimum event of its (launch, seed,
  * kernel, kind) slot, and the slot's event count.  tid_a/tid_b are global
- * linear thread ids (XB: block ids). */
+ * linear thread ids (XB: block ids).  key = launch (19 bits) | seed_idx (21) |
+ * kernel (4) | kind (4) | round (16; 0xFFFF for MISMATCH / XB). */
 typedef struct {
     uint64_t key, count;
     uint32_t kind, launch, seed_idx, kernel, round, site, array, addr, tid_a, tid_b, val_a, val_b;
@@ -123,6 +124,17 @@ int pg_load_ir(const char *text, size_t len, pg_ir **out);
  * (RACE: WW/RW/XB; OOB: out-of-bounds and uninitialised reads; BANK/COALESCE
  * report-only).  Enqueues on sp->cuda_stream. */
 int pg_check_equiv(const pg_ir *src, const pg_ir *tgt, const pg_space *sp, pg_run **out);
+
+/* N-kernel comparative assertion (SURVEY.md §8(d) C2 design: reduce0..6 pairwise): nk
+ * kernels (2..8), kernel k with launch list launches[k] (n_launch points each, the same
+ * parameter n in the same order; NULL entry or NULL array = sp->launch_src), each evaluated
+ * ONCE per (launch, seed), then every pair i < j compared on every global array that is
+ * out/inout in either (matched by name).  A mismatch of the pair (i, j) is an event of kernel
+ * i's MISMATCH slot with site = j (the slot's record is the minimum over j, X16; its count
+ * sums the mismatching cells of every pair).  Races / OOB / LIMIT per kernel as in
+ * pg_check_equiv.  BANK / COALESCE / LOCKSTEP are PG_E_ARG (pair checks). */
+int pg_check_equiv_n(const pg_ir *const *ks, uint32_t nk, const pg_launch *const *launches, const pg_space *sp,
+                     pg_run **out);
 
 /* Race premise of the key observation (L516-L520, L660-L662) for one kernel:
  * WW / RW / XB / OOB (and LIMIT) over the space; checks = RACE|OOB regardless

@@ -74,6 +74,12 @@ def lib():
                                       ctypes.POINTER(OrRec), ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64),
                                       ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64),
                                       ctypes.POINTER(ctypes.c_uint64)]
+            _lib.or_check_n.restype = ctypes.c_int
+            _lib.or_check_n.argtypes = [ctypes.POINTER(ctypes.c_char_p), ctypes.c_uint32,
+                                        ctypes.POINTER(ctypes.POINTER(OrLaunch)), ctypes.POINTER(OrSpace),
+                                        ctypes.POINTER(OrRec), ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64),
+                                        ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64),
+                                        ctypes.POINTER(ctypes.c_uint64)]
             _lib.or_exec.restype = ctypes.c_int
             _lib.or_exec.argtypes = [ctypes.c_char_p, ctypes.POINTER(OrLaunch), ctypes.c_uint64, ctypes.c_uint32,
                                      ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
@@ -158,6 +164,36 @@ def check(src: str, tgt, launch_src, launch_tgt=None, *, n_seeds=1, seed_base=0,
     out = [tuple(getattr(recs[i], f) for f in REC_FIELDS) for i in range(m)]
     return {"records": out, "n_records": n.value, "counts": list(counts), "first_key": list(first),
             "site_stats": stats}
+
+
+def check_n(texts, launches, *, n_seeds=1, seed_base=0, rank=0, world=1, input_mode=0, input_range=0, bits=32,
+            checks=EQUIV | RACE | OOB, wmax=32, cap=1 << 16):
+    """N-kernel check (or_check_n): every kernel once per (launch, seed), every pair i < j
+    compared, a pair's mismatch in kernel i's MISMATCH slot with site = j.  launches[k] is
+    kernel k's launch list.  Same result dict as check()."""
+    L = lib()
+    nk = len(texts)
+    arrs = [_launch_array(ls) for ls in launches]
+    ptrs = (ctypes.POINTER(OrLaunch) * nk)(*[ctypes.cast(a, ctypes.POINTER(OrLaunch)) for a in arrs])
+    tx = (ctypes.c_char_p * nk)(*[t.encode() for t in texts])
+    sp = OrSpace()
+    sp.launch_src = ptrs[0]
+    sp.launch_tgt = None
+    sp.n_launch = len(launches[0])
+    sp.seed_base, sp.n_seeds, sp.rank, sp.world = seed_base, n_seeds, rank, world
+    sp.input_mode, sp.input_range, sp.bits = input_mode, input_range, bits
+    sp.checks, sp.wmax, sp.mode = checks, wmax, MODE_EQUIV
+    recs = (OrRec * cap)()
+    n = ctypes.c_uint64(0)
+    counts = (ctypes.c_int64 * 16)()
+    first = (ctypes.c_int64 * 11)()
+    rc = L.or_check_n(tx, nk, ptrs, ctypes.byref(sp), recs, cap, ctypes.byref(n), counts, first, None)
+    if rc != 0:
+        raise OracleError(rc, L.or_last_error().decode())
+    m = min(n.value, cap)
+    out = [tuple(getattr(recs[i], f) for f in REC_FIELDS) for i in range(m)]
+    return {"records": out, "n_records": n.value, "counts": list(counts), "first_key": list(first),
+            "site_stats": None}
 
 
 def exec_kernel(text: str, launch, seed: int, *, input_mode=0, input_range=0, bits=32, checks=EQUIV | RACE | OOB,
@@ -276,3 +312,26 @@ def check_parallel(src: str, tgt, launch_src, launch_tgt=None, *, processes=0, *
                 stats[..., c] += s[..., c]
     return {"records": recs, "n_records": sum(p["n_records"] for p in parts), "counts": counts,
             "first_key": first, "site_stats": stats}
+
+
+def _check_n_shard(args):
+    texts, launches, kw, rank, world = args
+    return check_n(texts, launches, rank=rank, world=world, **kw)
+
+
+def check_n_parallel(texts, launches, *, processes=0, **kw):
+    """check_n() over host cores by seed shard, merged like check_parallel()."""
+    import multiprocessing as mp
+    n_seeds = kw.get("n_seeds", 1)
+    world = max(1, min(processes or len(os.sched_getaffinity(0)), n_seeds))
+    build()
+    if world == 1:
+        return check_n(texts, launches, **kw)
+    launches = [[tuple(map(tuple, (l.gdim, l.bdim, l.scalars))) if hasattr(l, "gdim") else l for l in ls]
+                for ls in launches]
+    with mp.get_context("fork").Pool(world) as pool:
+        parts = pool.map(_check_n_shard, [(texts, launches, kw, r, world) for r in range(world)])
+    recs = sorted((r for p in parts for r in p["records"]), key=lambda r: r[0])
+    return {"records": recs, "n_records": sum(p["n_records"] for p in parts),
+            "counts": [sum(p["counts"][i] for p in parts) for i in range(16)],
+            "first_key": [min(p["first_key"][i] for p in parts) for i in range(11)], "site_stats": None}

@@ -960,9 +960,9 @@ struct Rec {
     uint32_t kind, launch, seed_idx, kernel, round, site, array, addr, tid_a, tid_b, val_a, val_b;
 };
 
-/* X16: key = launch(19) | seed_idx(24) | kernel(1) | kind(4) | round(16) */
+/* X16: key = launch(19) | seed_idx(21) | kernel(4) | kind(4) | round(16) */
 static uint64_t make_key(uint32_t launch, uint32_t seed_idx, uint32_t kernel, uint32_t kind, uint32_t round) {
-    return ((uint64_t)launch << 45) | ((uint64_t)seed_idx << 21) | ((uint64_t)kernel << 20) |
+    return ((uint64_t)launch << 45) | ((uint64_t)seed_idx << 24) | ((uint64_t)kernel << 20) |
            ((uint64_t)kind << 16) | (uint64_t)(round & 0xFFFFu);
 }
 
@@ -1127,8 +1127,8 @@ struct Results {
     /* slots[(launch, seed_j, kernel)][kind] */
     std::map<std::tuple<uint32_t, uint32_t, uint32_t>, SlotSet> slots;
     uint64_t instances = 0;
-    std::vector<uint64_t> site_stats;   /* [n_launch][2][max_sites][8] */
-    uint32_t max_sites = 0;
+    std::vector<uint64_t> site_stats;   /* [n_launch][stats_nk][max_sites][8] */
+    uint32_t max_sites = 0, stats_nk = 2;
     std::vector<DFRow> df;
     std::vector<Snap> snaps[2];      /* per kernel, this instance */
     std::vector<DivRow> div;
@@ -1477,7 +1477,7 @@ struct Exec {
             const Arr& A = K.arrs[(size_t)a];
             uint64_t* st = nullptr;
             if (site < (int)res.max_sites)
-                st = &res.site_stats[(((size_t)launch_idx * 2 + kernel_idx) * res.max_sites + (size_t)site) * 8];
+                st = &res.site_stats[(((size_t)launch_idx * res.stats_nk + kernel_idx) * res.max_sites + (size_t)site) * 8];
             if (A.space == SP_SHARED) {
                 if (!(cfg.checks & CHK_BANK)) continue;
                 uint32_t nb = cfg.bank_model == 1 ? 16u : 32u;
@@ -1746,11 +1746,16 @@ static void lockstep_compare(const Kernel& ks, uint32_t li, uint32_t sj, Results
     if (found) res.div.push_back(best);
 }
 
-static void run_space(const Kernel* ks, const Kernel* kt, const Space& S, Results& res) {
-    KInfo ki[2];
-    const Kernel* kk[2] = {ks, kt};
-    int nk = kt ? 2 : 1;
-    /* X8: global ids = index in the sorted union of both kernels' global-array names */
+/* The kernels of one check over the space: each is run once per (launch, seed); with two
+ * or more, the comparative assertion (L441-L444, L652-L657) on every pair i < j, over every
+ * global array that is out/inout in either kernel (matched by name).  A mismatch of the pair
+ * is an event in slot (instance, kernel i, MISMATCH); its site field names j in N-kernel
+ * checks (nmode) and is NONE for the two-kernel check. */
+static void run_space(const std::vector<const Kernel*>& kk, const std::vector<const Launch*>& lists, const Space& S,
+                      Results& res, bool nmode) {
+    const int nk = (int)kk.size();
+    std::vector<KInfo> ki((size_t)nk);
+    /* X8: global ids = index in the sorted union of the kernels' global-array names */
     std::vector<std::string> names;
     for (int k = 0; k < nk; k++)
         for (auto& A : kk[k]->arrs) if (A.space == SP_GLOBAL) names.push_back(A.name);
@@ -1768,12 +1773,15 @@ static void run_space(const Kernel* ks, const Kernel* kt, const Space& S, Result
                 ki[k].gid[a] = (int)(std::lower_bound(names.begin(), names.end(), kk[k]->arrs[a].name) - names.begin());
     }
     for (uint32_t li = 0; li < S.n_launch; li++) {
-        const Launch* LL[2] = {&S.launch_src[li], S.launch_tgt ? &S.launch_tgt[li] : &S.launch_src[li]};
-        for (int k = 0; k < nk; k++) check_launch(*kk[k], *LL[k]);
+        std::vector<const Launch*> LL((size_t)nk);
+        for (int k = 0; k < nk; k++) {
+            LL[k] = &lists[k][li];
+            check_launch(*kk[k], *LL[k]);
+        }
         for (uint32_t sj = S.rank; sj < S.n_seeds; sj += S.world) {
             uint64_t seed = S.seed_base + sj;
-            std::vector<std::vector<uint32_t>> fin[2], flast[2], fsize[2];
-            std::vector<uint32_t> fsz[2];
+            std::vector<std::vector<std::vector<uint32_t>>> fin((size_t)nk), flast((size_t)nk);
+            std::vector<std::vector<uint32_t>> fsz((size_t)nk);
             res.snaps[0].clear();
             res.snaps[1].clear();
             for (int k = 0; k < nk; k++) {
@@ -1784,26 +1792,28 @@ static void run_space(const Kernel* ks, const Kernel* kt, const Space& S, Result
                 flast[k] = ex.glast;
                 fsz[k] = ex.size;
             }
-            if (nk == 2 && S.cfg.lock_rounds) lockstep_compare(*ks, li, sj, res);
-            if (nk == 2 && (S.cfg.checks & CHK_EQUIV)) {
-                /* comparative assertion o_s = o_t (L441-L444, L652-L657) */
-                Slot* sl = res.slots[std::make_tuple(li, sj, 0u)].s;
-                for (size_t as = 0; as < ks->arrs.size(); as++) {
-                    const Arr& A = ks->arrs[as];
-                    if (A.space != SP_GLOBAL) continue;
-                    for (size_t at_ = 0; at_ < kt->arrs.size(); at_++) {
-                        const Arr& B = kt->arrs[at_];
-                        if (B.space != SP_GLOBAL || B.name != A.name) continue;
-                        if (A.mode == M_IN && B.mode == M_IN) continue;
-                        uint32_t n = std::min(fsz[0][as], fsz[1][at_]);
-                        for (uint32_t i = 0; i < n; i++) {
-                            uint32_t va = fin[0][as][i], vb = fin[1][at_][i];
-                            if (va != vb) {
-                                Ev e;
-                                uint32_t f[8] = {ROUND_END, (uint32_t)ki[0].gid[as], i, flast[0][as][i] - 1,
-                                                 flast[1][at_][i] - 1, NONE32, va, vb};
-                                memcpy(e.f, f, sizeof f);
-                                sl[K_MISMATCH].add(e);
+            if (nk == 2 && S.cfg.lock_rounds) lockstep_compare(*kk[0], li, sj, res);
+            if (nk < 2 || !(S.cfg.checks & CHK_EQUIV)) continue;
+            for (int i = 0; i < nk; i++) {
+                Slot* sl = res.slots[std::make_tuple(li, sj, (uint32_t)i)].s;
+                for (int j = i + 1; j < nk; j++) {
+                    for (size_t as = 0; as < kk[i]->arrs.size(); as++) {
+                        const Arr& A = kk[i]->arrs[as];
+                        if (A.space != SP_GLOBAL) continue;
+                        for (size_t at_ = 0; at_ < kk[j]->arrs.size(); at_++) {
+                            const Arr& B = kk[j]->arrs[at_];
+                            if (B.space != SP_GLOBAL || B.name != A.name) continue;
+                            if (A.mode == M_IN && B.mode == M_IN) continue;
+                            uint32_t n = std::min(fsz[i][as], fsz[j][at_]);
+                            for (uint32_t c = 0; c < n; c++) {
+                                uint32_t va = fin[i][as][c], vb = fin[j][at_][c];
+                                if (va != vb) {
+                                    Ev e;
+                                    uint32_t f[8] = {ROUND_END, (uint32_t)ki[i].gid[as], c, flast[i][as][c] - 1,
+                                                     flast[j][at_][c] - 1, nmode ? (uint32_t)j : NONE32, va, vb};
+                                    memcpy(e.f, f, sizeof f);
+                                    sl[K_MISMATCH].add(e);
+                                }
                             }
                         }
                     }
@@ -1846,27 +1856,32 @@ static thread_local std::string or_err;
 
 const char* or_last_error(void) { return or_err.c_str(); }
 
-/* Check a pair (tgt != NULL) or a single kernel over the space.
- * recs: caller buffer of cap records (canonical order); counts[16]; first_key[11];
- * site_stats: NULL or uint64[n_launch][2][max_sites][8] =
- *   [space (1 shared, 2 global), warp-accesses, conflicted|uncoalesced, max degree|sectors,
- *    sum degree|sectors, sum ideal, sum active lanes, 0]. */
-int or_check(const char* src, const char* tgt, const or_space* sp, or_rec* recs, uint64_t cap, uint64_t* n_recs,
-             int64_t* counts, int64_t* first_key, uint64_t* site_stats) {
+/* The kernels texts[0..nk) over the space, the launches of kernel k in lists[k] (shared by
+ * or_check and or_check_n). */
+static int check_common(const char* const* texts, uint32_t nk, const or_launch* const* lists, bool nmode,
+                        const or_space* sp, or_rec* recs, uint64_t cap, uint64_t* n_recs, int64_t* counts,
+                        int64_t* first_key, uint64_t* site_stats) {
     using namespace orc;
     try {
-        if (!src || !sp || !n_recs || !counts || !first_key) throw Error(E_ARG, "null argument");
+        if (!texts || !sp || !n_recs || !counts || !first_key || nk < 1 || nk > 8) throw Error(E_ARG, "null argument");
+        for (uint32_t k = 0; k < nk; k++)
+            if (!texts[k]) throw Error(E_ARG, "null kernel");
         if (sp->world == 0 || sp->rank >= sp->world) throw Error(E_ARG, "bad rank/world");
         if (sp->bits < 1 || sp->bits > 32) throw Error(E_ARG, "bits must be 1..32");
         if (sp->n_launch >= (1u << 18)) throw Error(E_LIMIT, "too many launches");
-        if (sp->n_seeds >= (1u << 24)) throw Error(E_LIMIT, "too many seeds");
-        std::unique_ptr<Kernel> ks = parse_kernel(src);
-        std::unique_ptr<Kernel> kt;
-        if (tgt) kt = parse_kernel(tgt);
-        Space S;
+        if (sp->n_seeds >= (1u << 21)) throw Error(E_LIMIT, "too many seeds");
+        std::vector<std::unique_ptr<Kernel>> ks;
+        std::vector<const Kernel*> kk;
+        std::vector<const Launch*> ll;
         static_assert(sizeof(or_launch) == sizeof(Launch), "launch layout");
-        S.launch_src = reinterpret_cast<const Launch*>(sp->launch_src);
-        S.launch_tgt = reinterpret_cast<const Launch*>(sp->launch_tgt);
+        for (uint32_t k = 0; k < nk; k++) {
+            ks.push_back(parse_kernel(texts[k]));
+            kk.push_back(ks.back().get());
+            ll.push_back(reinterpret_cast<const Launch*>(lists[k]));
+        }
+        Space S;
+        S.launch_src = ll[0];
+        S.launch_tgt = nk > 1 ? ll[1] : nullptr;
         S.n_launch = sp->n_launch;
         S.seed_base = sp->seed_base;
         S.n_seeds = sp->n_seeds;
@@ -1882,8 +1897,9 @@ int or_check(const char* src, const char* tgt, const or_space* sp, or_rec* recs,
         S.mode = sp->mode;
         Results res;
         res.max_sites = site_stats ? sp->max_sites : 0;
-        res.site_stats.assign((size_t)sp->n_launch * 2 * res.max_sites * 8, 0);
-        run_space(ks.get(), kt.get(), S, res);
+        res.stats_nk = std::max<uint32_t>(2, nk);
+        res.site_stats.assign((size_t)sp->n_launch * res.stats_nk * res.max_sites * 8, 0);
+        run_space(kk, ll, S, res, nmode);
         for (int i = 0; i < 16; i++) counts[i] = 0;
         for (int i = 0; i < 11; i++) first_key[i] = INT64_MAX;
         counts[0] = (int64_t)res.instances;
@@ -1924,6 +1940,29 @@ int or_check(const char* src, const char* tgt, const or_space* sp, or_rec* recs,
         or_err = e.what();
         return -1;
     }
+}
+
+/* Check a pair (tgt != NULL) or a single kernel over the space.
+ * recs: caller buffer of cap records (canonical order); counts[16]; first_key[11];
+ * site_stats: NULL or uint64[n_launch][2][max_sites][8] =
+ *   [space (1 shared, 2 global), warp-accesses, conflicted|uncoalesced, max degree|sectors,
+ *    sum degree|sectors, sum ideal, sum active lanes, 0]. */
+int or_check(const char* src, const char* tgt, const or_space* sp, or_rec* recs, uint64_t cap, uint64_t* n_recs,
+             int64_t* counts, int64_t* first_key, uint64_t* site_stats) {
+    if (!sp) return -1;
+    const char* texts[2] = {src, tgt};
+    const or_launch* lists[2] = {sp->launch_src, sp->launch_tgt ? sp->launch_tgt : sp->launch_src};
+    return check_common(texts, tgt ? 2u : 1u, lists, false, sp, recs, cap, n_recs, counts, first_key, site_stats);
+}
+
+/* N-kernel check (nk in 1..8): every kernel once per (launch, seed), launches[k] its launch
+ * list (n_launch each, the same points n); the comparative assertion on every pair i < j,
+ * MISMATCH records in the slot of kernel i with site = j.  site_stats: [n_launch][max(2,nk)]
+ * [max_sites][8]. */
+int or_check_n(const char* const* texts, uint32_t nk, const or_launch* const* launches, const or_space* sp,
+               or_rec* recs, uint64_t cap, uint64_t* n_recs, int64_t* counts, int64_t* first_key,
+               uint64_t* site_stats) {
+    return check_common(texts, nk, launches, true, sp, recs, cap, n_recs, counts, first_key, site_stats);
 }
 
 /* Run one kernel for one launch/seed and return its initial and final global
@@ -2051,7 +2090,7 @@ int or_lockstep(const char* src, const char* tgt, const or_space* sp, uint32_t l
         S.cfg.lock_rounds = lock_rounds;
         S.mode = sp->mode;
         Results res;
-        run_space(ks.get(), kt.get(), S, res);
+        run_space({ks.get(), kt.get()}, {S.launch_src, S.launch_tgt ? S.launch_tgt : S.launch_src}, S, res, false);
         *n_rows = res.div.size();
         for (size_t i = 0; i < res.div.size() && i < cap_rows; i++) memcpy(rows + i * 10, &res.div[i], sizeof(DivRow));
         return 0;

@@ -56,16 +56,15 @@ __device__ __forceinline__ u32 fill_value(u32 op, u32 mode, u32 range, u32 mask,
     return v & mask;
 }
 __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ jobs, u32 n_jobs, u32 task_base,
-                                                     u32 n_tasks, u32* arena_s, u32* arena_t, u32* input,
-                                                     u64 seed_base, u32 mode, u32 range, u32 mask,
-                                                     const u32* flags, const u32* any) {
+                                                     u32 n_tasks, const PgRegions R, u64 seed_base, u32 mode,
+                                                     u32 range, u32 mask, const u32* flags, const u32* any) {
     if (flags && !*any) return;   // re-initialisation with nothing flagged
     __shared__ u32 s_job;
     if (threadIdx.x == 0) s_job = 0u;
     for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
         const PgFill f = jobs[pg_task_job(jobs, n_jobs, task_base, task, &s_job)];
         const u32 lt = task - (f.task0 - task_base);
-        u32* region = f.target == 0 ? arena_s : f.target == 1 ? arena_t : input;
+        u32* region = R.r[f.target];
         if (f.n > PG_FILL_SMALL) {
             const u32 nch = (f.n + PG_FILL_CHUNK - 1u) / PG_FILL_CHUNK;
             const u32 inst = lt / nch, w0 = (lt - inst * nch) * PG_FILL_CHUNK;
@@ -98,13 +97,11 @@ __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ 
     }
 }
 
-__device__ __forceinline__ u32 cmp_val(const u32* region, u32 kind, u64 off, u32 i) { return region[off + i]; }
-
-// K3a: count mismatching cells per (instance, array); keep the minimum (gid, addr)
-// per instance.  One CTA task per grid-stride step (pg_task_job).
+// K3a: count mismatching cells per (instance, pair, array); keep the minimum (gid, addr) per
+// (instance, kernel i) - the pairs (i, j) of an N-kernel check share kernel i's MISMATCH slot.
+// One CTA task per grid-stride step (pg_task_job).
 __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs, u32 n_jobs, u32 n_tasks,
-                                                  const u32* arena_s, const u32* arena_t, const u32* input,
-                                                  PgSlot* slots, u64* mm_key) {
+                                                  const PgRegions R, PgSlot* slots, u64* mm_key) {
     __shared__ u32 s_cnt;
     __shared__ u32 s_min;
     __shared__ u32 s_job;
@@ -112,21 +109,21 @@ __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs
     for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
         const PgCmp c = jobs[pg_task_job(jobs, n_jobs, 0u, task, &s_job)];
         const u32 lt = task - c.task0;
-        const u32* rs = c.src_kind == 0 ? arena_s : input;
-        const u32* rt = c.tgt_kind == 0 ? arena_t : input;
+        const u32* rs = R.r[c.src_r];
+        const u32* rt = R.r[c.tgt_r];
         if (c.n <= PG_FILL_SMALL) {   // a warp per instance
             const u32 inst = lt * 8u + (threadIdx.x >> 5), lane = threadIdx.x & 31u;
             if (inst >= c.n_inst) continue;
             const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
             u32 cnt = 0, mn = PG_NEVER;
             for (u32 i = lane; i < c.n; i += 32u) {
-                if (cmp_val(rs, c.src_kind, so, i) != cmp_val(rt, c.tgt_kind, to, i)) { cnt++; mn = min(mn, i); }
+                if (rs[so + i] != rt[to + i]) { cnt++; mn = min(mn, i); }
             }
             cnt = __reduce_add_sync(0xffffffffu, cnt);
             mn = __reduce_min_sync(0xffffffffu, mn);
             if (lane == 0 && cnt) {
                 atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step].count, (u64)cnt);
-                atomicMin(&mm_key[c.inst0 + inst], ((u64)c.gid << 32) | mn);
+                atomicMin(&mm_key[c.mm0 + (u64)inst * c.mm_step], ((u64)c.gid << 32) | mn);
             }
             continue;
         }
@@ -137,7 +134,7 @@ __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs
         const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
         u32 cnt = 0, mn = PG_NEVER;
         for (u32 i = w0 + threadIdx.x; i < w1; i += blockDim.x) {
-            if (cmp_val(rs, c.src_kind, so, i) != cmp_val(rt, c.tgt_kind, to, i)) { cnt++; mn = min(mn, i); }
+            if (rs[so + i] != rt[to + i]) { cnt++; mn = min(mn, i); }
         }
         cnt = __reduce_add_sync(0xffffffffu, cnt);
         mn = __reduce_min_sync(0xffffffffu, mn);
@@ -145,34 +142,60 @@ __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs
         __syncthreads();
         if (threadIdx.x == 0 && s_cnt) {
             atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step].count, (u64)s_cnt);
-            atomicMin(&mm_key[c.inst0 + inst], ((u64)c.gid << 32) | s_min);
+            atomicMin(&mm_key[c.mm0 + (u64)inst * c.mm_step], ((u64)c.gid << 32) | s_min);
         }
         __syncthreads();
     }
 }
 
-// K3b: fill the MISMATCH record of every failing instance from its minimum cell.
-__global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__ jobs, const u32* arena_s,
-                                                       const u32* arena_t, const u32* input, PgSlot* slots,
-                                                       const u64* mm_key) {
+__device__ __forceinline__ u32 pg_cmp_lw(const PgRegions& R, u32 r, u64 lw, u64 inst, u64 stride, u32 addr) {
+    return r == PG_R_INPUT ? PG_NEVER : R.r[r][lw + inst * stride + addr] - 1u;
+}
+
+// K3b: among the pairs (i, j) that mismatch at kernel i's minimum cell, the minimum
+// (tid_b, site) - the remaining fields of the X16 minimum event.
+__global__ void __launch_bounds__(128) pg_compare_pick(const PgCmp* __restrict__ jobs, const PgRegions R,
+                                                       const u64* mm_key, u64* mm2) {
     const PgCmp c = jobs[blockIdx.y];
     const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
     if (inst >= c.n_inst) return;
-    const u64 k = mm_key[c.inst0 + inst];
+    const u64 mi = c.mm0 + (u64)inst * c.mm_step;
+    const u64 k = mm_key[mi];
     if (k == ~0ull || (u32)(k >> 32) != c.gid) return;
     const u32 addr = (u32)k;
-    const u32* rs = c.src_kind == 0 ? arena_s : input;
-    const u32* rt = c.tgt_kind == 0 ? arena_t : input;
-    const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
+    if (addr >= c.n) return;
+    const u32 a = R.r[c.src_r][c.src_off + (u64)inst * c.src_stride + addr];
+    const u32 b = R.r[c.tgt_r][c.tgt_off + (u64)inst * c.tgt_stride + addr];
+    if (a == b) return;
+    const u32 tb = pg_cmp_lw(R, c.tgt_r, c.tgt_lw, inst, c.tgt_stride, addr);
+    atomicMin(&mm2[mi], ((u64)tb << 32) | c.site);
+}
+
+// K3c: fill the MISMATCH record of every failing (instance, kernel i) from the pair the
+// pick chose.
+__global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__ jobs, const PgRegions R,
+                                                       PgSlot* slots, const u64* mm_key, const u64* mm2) {
+    const PgCmp c = jobs[blockIdx.y];
+    const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
+    if (inst >= c.n_inst) return;
+    const u64 mi = c.mm0 + (u64)inst * c.mm_step;
+    const u64 k = mm_key[mi];
+    if (k == ~0ull || (u32)(k >> 32) != c.gid) return;
+    const u32 addr = (u32)k;
+    if (addr >= c.n) return;
+    const u32 a = R.r[c.src_r][c.src_off + (u64)inst * c.src_stride + addr];
+    const u32 b = R.r[c.tgt_r][c.tgt_off + (u64)inst * c.tgt_stride + addr];
+    const u32 tb = pg_cmp_lw(R, c.tgt_r, c.tgt_lw, inst, c.tgt_stride, addr);
+    if (a == b || mm2[mi] != (((u64)tb << 32) | c.site)) return;
     PgSlot* s = &slots[c.slot0 + (u64)inst * c.slot_step];
     s->f[0] = 0xFFFFu;
     s->f[1] = c.gid;
     s->f[2] = addr;
-    s->f[3] = c.src_kind == 0 ? arena_s[c.src_lw + (u64)inst * c.src_stride + addr] - 1u : PG_NEVER;
-    s->f[4] = c.tgt_kind == 0 ? arena_t[c.tgt_lw + (u64)inst * c.tgt_stride + addr] - 1u : PG_NEVER;
-    s->f[5] = PG_NEVER;
-    s->f[6] = cmp_val(rs, c.src_kind, so, addr);
-    s->f[7] = cmp_val(rt, c.tgt_kind, to, addr);
+    s->f[3] = pg_cmp_lw(R, c.src_r, c.src_lw, inst, c.src_stride, addr);
+    s->f[4] = tb;
+    s->f[5] = c.site;
+    s->f[6] = a;
+    s->f[7] = b;
     s->has = 1u;
 }
 
@@ -337,19 +360,19 @@ __device__ __forceinline__ bool kind_failing(u32 kind, u32 banks_mode) {
 // K4a: per instance (launch, local seed m): count non-empty slots, fold counts
 // and keys into the summary (X16/X17).
 __global__ void __launch_bounds__(256) pg_summarize(const PgSlot* __restrict__ slots, u32 n_inst, u32 n_local,
-                                                    u32 rank, u32 world, u32 banks_mode, u32* inst_nrec,
+                                                    u32 rank, u32 world, u32 banks_mode, u32 nks, u32* inst_nrec,
                                                     long long* first_key, long long* counts) {
     const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
     if (inst >= n_inst) return;
     const u32 li = inst / n_local, m = inst % n_local;
     const u32 sj = rank + m * world;
     u32 n = 0, failing = 0;
-    for (u32 k = 0; k < 2; k++) {
+    for (u32 k = 0; k < nks; k++) {
         for (u32 kind = 0; kind < PG_NK; kind++) {
-            const PgSlot& s = slots[((u64)inst * 2 + k) * PG_NK + kind];
+            const PgSlot& s = slots[((u64)inst * nks + k) * PG_NK + kind];
             if (s.count == 0 || !s.has) continue;
             n++;
-            const long long key = (long long)(((u64)li << 45) | ((u64)sj << 21) | ((u64)k << 20) |
+            const long long key = (long long)(((u64)li << 45) | ((u64)sj << 24) | ((u64)k << 20) |
                                               ((u64)kind << 16) | (u64)(s.f[0] & 0xFFFFu));
             atomicAdd((unsigned long long*)&counts[1 + kind], (unsigned long long)s.count);
             atomicMin(&first_key[1 + kind], key);
@@ -407,21 +430,21 @@ struct PgCexDev {
 // The run's record count (its own records, before any cross-rank reduction of the counters)
 // goes to *total.
 __global__ void __launch_bounds__(256) pg_compact(const PgSlot* __restrict__ slots, u32 n_inst, u32 n_local,
-                                                  u32 rank, u32 world, const u32* inst_nrec, const u64* offsets,
-                                                  PgCexDev* out, u64 cap, u64* total) {
+                                                  u32 rank, u32 world, u32 nks, const u32* inst_nrec,
+                                                  const u64* offsets, PgCexDev* out, u64 cap, u64* total) {
     const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
     if (inst == 0) *total = offsets[n_inst - 1] + inst_nrec[n_inst - 1];
     if (inst >= n_inst) return;
     const u32 li = inst / n_local, m = inst % n_local;
     const u32 sj = rank + m * world;
     u64 o = offsets[inst];
-    for (u32 k = 0; k < 2; k++) {
+    for (u32 k = 0; k < nks; k++) {
         for (u32 kind = 0; kind < PG_NK; kind++) {
-            const PgSlot& s = slots[((u64)inst * 2 + k) * PG_NK + kind];
+            const PgSlot& s = slots[((u64)inst * nks + k) * PG_NK + kind];
             if (s.count == 0 || !s.has) continue;
             if (o < cap) {
                 PgCexDev r;
-                r.key = ((u64)li << 45) | ((u64)sj << 21) | ((u64)k << 20) | ((u64)kind << 16) | (u64)(s.f[0] & 0xFFFFu);
+                r.key = ((u64)li << 45) | ((u64)sj << 24) | ((u64)k << 20) | ((u64)kind << 16) | (u64)(s.f[0] & 0xFFFFu);
                 r.count = s.count;
                 r.kind = kind;
                 r.launch = li;
@@ -530,13 +553,13 @@ u32 sm_count() {
 u32 task_grid(u32 n_tasks) { return n_tasks < sm_count() * 16u ? n_tasks : sm_count() * 16u; }
 
 
-cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 task_base, u32 n_tasks, u32* arena_s, u32* arena_t,
-                       u32* input, u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags,
+cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 task_base, u32 n_tasks, const PgRegions& R,
+                       u64 seed_base, u32 mode, u32 range, u32 mask, cudaStream_t st, const u32* flags,
                        const u32* any) {
     if (!n_jobs || !n_tasks) return cudaSuccess;
     const u32 grid = task_grid(n_tasks);
-    pg_gen_inputs<<<grid, 256, 0, st>>>(jobs, n_jobs, task_base, n_tasks, arena_s, arena_t, input, seed_base, mode,
-                                        range, mask, flags, any);
+    pg_gen_inputs<<<grid, 256, 0, st>>>(jobs, n_jobs, task_base, n_tasks, R, seed_base, mode, range, mask, flags,
+                                        any);
     return cudaGetLastError();
 }
 
@@ -553,15 +576,19 @@ cudaError_t count_reduce(const u64* inst_cnt, u32 n, long long* counts, cudaStre
     return cudaGetLastError();
 }
 
-cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 n_tasks, u32 max_inst, const u32* arena_s,
-                    const u32* arena_t, const u32* input, PgSlot* slots, u64* mm_key, cudaStream_t st) {
+cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 n_tasks, u32 max_inst, const PgRegions& R, PgSlot* slots,
+                    u64* mm_key, u64* mm2, cudaStream_t st) {
     if (!n_jobs) return cudaSuccess;
-    pg_compare<<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, arena_s, arena_t,
-                                                                            input, slots, mm_key);
+    pg_compare<<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, R, slots, mm_key);
     for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
         const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
         dim3 g2((max_inst + 127) / 128, nj);
-        pg_compare_fill<<<g2, 128, 0, st>>>(jobs + j0, arena_s, arena_t, input, slots, mm_key);
+        pg_compare_pick<<<g2, 128, 0, st>>>(jobs + j0, R, mm_key, mm2);
+    }
+    for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
+        const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
+        dim3 g2((max_inst + 127) / 128, nj);
+        pg_compare_fill<<<g2, 128, 0, st>>>(jobs + j0, R, slots, mm_key, mm2);
     }
     return cudaGetLastError();
 }
@@ -611,18 +638,19 @@ cudaError_t reset_counters(long long* first_key, long long* counts, cudaStream_t
 }
 
 cudaError_t summarize_scan(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, u32 banks_mode,
-                           u32* inst_nrec, u64* offsets, long long* first_key, long long* counts, cudaStream_t st) {
+                           u32 nks, u32* inst_nrec, u64* offsets, long long* first_key, long long* counts,
+                           cudaStream_t st) {
     if (!n_inst) return cudaSuccess;
-    pg_summarize<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, banks_mode, inst_nrec,
-                                                       first_key, counts);
+    pg_summarize<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, banks_mode, nks,
+                                                       inst_nrec, first_key, counts);
     pg_scan<<<1, 1024, 0, st>>>(inst_nrec, offsets, n_inst);
     return cudaGetLastError();
 }
 
-cudaError_t compact(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, const u32* inst_nrec,
-                    const u64* offsets, void* out, u64 cap, u64* total, cudaStream_t st) {
+cudaError_t compact(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, u32 nks,
+                    const u32* inst_nrec, const u64* offsets, void* out, u64 cap, u64* total, cudaStream_t st) {
     if (!n_inst) return cudaSuccess;
-    pg_compact<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, inst_nrec, offsets,
+    pg_compact<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, nks, inst_nrec, offsets,
                                                      (PgCexDev*)out, cap, total);
     return cudaGetLastError();
 }

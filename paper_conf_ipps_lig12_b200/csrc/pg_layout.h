@@ -15,6 +15,13 @@ typedef unsigned short u16;
 #define PG_NEVER 0xFFFFFFFFu
 #define PG_NK 10
 #define PG_MAXARR 16
+#define PG_MAXK 8          // kernels of one check (pg_check_equiv_n)
+#define PG_R_INPUT PG_MAXK  // region index of the input region (arenas are regions 0..PG_MAXK-1)
+
+// base pointers of the regions a K1 / K3 job addresses: arena of kernel k, then the input region
+struct PgRegions {
+    u32* r[PG_MAXK + 1];
+};
 
 enum { PGK_BARRIER_DIV = 0, PGK_OOB = 1, PGK_WW = 2, PGK_RW = 3, PGK_XB = 4, PGK_MISMATCH = 5, PGK_BANK = 6,
        PGK_UNCOAL = 7, PGK_UNINIT = 8, PGK_LIMIT = 9 };
@@ -122,7 +129,7 @@ struct PgFill {
     u32 op;       // PGF_*
     u32 gid;      // PRF tag (X8)
     u32 value;    // PGF_CONST fill value
-    u32 target;   // 0 arena (src), 1 arena (tgt), 2 input region
+    u32 target;   // region: arena of kernel k (0..PG_MAXK-1) or PG_R_INPUT
     u32 inst0;    // batch-local index of instance 0 (re-initialisation of flagged instances)
     u32 task0;    // first CTA task of this job in the batch's fill list (pg_fill_tasks)
     u32 istep;    // instances 0, istep, 2 istep, ... (n_inst of them): stamps that only the first
@@ -160,13 +167,16 @@ struct PgLock {
     u32 n_inst, nblocks, size, rounds, arr_slot, pad;
 };
 
-// K3 (pg_compare) job: one compared global array for n_inst consecutive
-// instances of one launch (H7).
+// K3 (pg_compare) job: one compared global array of one pair of kernels (i, j) for n_inst
+// consecutive instances of one launch (H7).
 struct PgCmp {
-    u64 src_off, tgt_off;        // u32-word offsets of instance 0: values in an arena (kind 0) or the input (kind 1)
+    u64 src_off, tgt_off;        // u32-word offsets of instance 0 in their regions
     u64 src_stride, tgt_stride;  // per-instance strides of the regions the offsets point into
-    u64 src_lw, tgt_lw;          // last-writer words of instance 0 (kind 0 only)
-    u64 slot0, slot_step;        // MISMATCH slot of (instance 0, kernel 0) and stride
-    u32 inst0, n_inst, gid, n, src_kind, tgt_kind;
-    u32 task0, pad;              // first CTA task (pg_fill_tasks(n, n_inst))
+    u64 src_lw, tgt_lw;          // last-writer words of instance 0 (arena regions only)
+    u64 slot0, slot_step;        // MISMATCH slot of (instance 0, kernel i) and stride
+    u32 inst0, n_inst, gid, n;
+    u32 src_r, tgt_r;            // regions: arena of kernel i / j, or PG_R_INPUT (array only read)
+    u32 task0;                   // first CTA task (pg_fill_tasks(n, n_inst))
+    u32 site;                    // record site field: j in N-kernel checks, PG_NEVER for a pair
+    u64 mm0, mm_step;            // per-(instance, kernel i) minimum-cell words of instance 0, stride
 };

@@ -37,5 +37,5 @@ def first_witness(first_key: int):
     """Decode the first-witness launch / seed index from a key (X16); None if no failure."""
     if first_key >= INT64_MAX:
         return None
-    return {"launch": first_key >> 45, "seed_idx": (first_key >> 21) & 0xFFFFFF, "kernel": (first_key >> 20) & 1,
+    return {"launch": first_key >> 45, "seed_idx": (first_key >> 24) & 0x1FFFFF, "kernel": (first_key >> 20) & 0xF,
             "kind": (first_key >> 16) & 0xF, "round": first_key & 0xFFFF}

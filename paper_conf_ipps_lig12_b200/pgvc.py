@@ -74,7 +74,7 @@ class PgError(RuntimeError):
 
 
 _lib = None
-EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
+EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
            "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_seed_oblivious",
            "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals", "pg_merge_counters",
            "pg_measure_int32_peak",
@@ -94,6 +94,8 @@ def lib():
     L.pg_load_ir.argtypes = [ctypes.c_char_p, ctypes.c_size_t, ctypes.POINTER(vp)]
     L.pg_check_equiv.argtypes = [vp, vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_check_races.argtypes = [vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
+    L.pg_check_equiv_n.argtypes = [ctypes.POINTER(vp), ctypes.c_uint32, ctypes.POINTER(ctypes.POINTER(PgLaunch)),
+                                   ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_check_banks.argtypes = [vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_check_property.argtypes = [vp, vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_collect_cex.argtypes = [vp, ctypes.POINTER(PgCex), ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t),
@@ -119,7 +121,7 @@ def lib():
     L.pg_version.restype = ctypes.c_char_p
     L.pg_ir_free.argtypes = [vp]
     L.pg_run_free.argtypes = [vp]
-    for f in ("pg_load_ir", "pg_check_equiv", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
+    for f in ("pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
               "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info",
               "pg_ir_seed_oblivious", "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals",
               "pg_merge_counters", "pg_measure_int32_peak"):
@@ -339,6 +341,33 @@ def pg_check_equiv(src: Ir, tgt: Ir, space: Space) -> Run:
     return _run(lib().pg_check_equiv, [src, tgt], space)
 
 
+def pg_check_equiv_n(kernels: Sequence[Ir], launches: Sequence[Sequence], space: Space) -> Run:
+    """Every kernel once per (launch, seed), every pair compared (pg_check_equiv_n).
+    launches[k]: kernel k's launch list (same length for all); space.launch_src is ignored
+    except as the list length / fallback (pass launches[0])."""
+    if not 2 <= len(kernels) <= 8 or len(launches) != len(kernels):
+        raise PgError(PG_E_ARG, "2 to 8 kernels, one launch list each")
+    n = len(launches[0])
+    if any(len(l) != n for l in launches):
+        raise PgError(PG_E_ARG, "launch lists of different lengths")
+    sp, keep = space.marshal()
+    key = (id(launches), len(launches), n)
+    cached = space.__dict__.get("_n_arrays")   # (marshalled once per Space object, as marshal() does)
+    if cached is not None and cached[0] == key:
+        arrs, ptrs = cached[1], cached[2]
+    else:
+        arrs = [(PgLaunch * max(1, n))(*[_launch(l) for l in ls]) for ls in launches]
+        ptrs = (ctypes.POINTER(PgLaunch) * len(arrs))(*[ctypes.cast(a, ctypes.POINTER(PgLaunch)) for a in arrs])
+        space.__dict__["_n_arrays"] = (key, arrs, ptrs)
+    sp.launch_src = ptrs[0]
+    sp.launch_tgt = None
+    sp.n_launch = n
+    hs = (ctypes.c_void_p * len(kernels))(*[k.handle.value for k in kernels])
+    h = ctypes.c_void_p()
+    _ck(lib().pg_check_equiv_n(hs, len(kernels), ptrs, ctypes.byref(sp), ctypes.byref(h)))
+    return Run(h, space, (keep, arrs, ptrs, kernels))
+
+
 def pg_check_races(k: Ir, space: Space) -> Run:
     return _run(lib().pg_check_races, [k], space)
 
@@ -355,6 +384,7 @@ def pg_check_property(k: Ir, post: Ir, space: Space) -> Run:
 
 
 check_equiv, check_races, check_banks, check_property = pg_check_equiv, pg_check_races, pg_check_banks, pg_check_property
+check_equiv_n = pg_check_equiv_n
 
 
 def merge_counters(first_keys, counts, out_first_key, out_counts, stream: int = 0):

@@ -143,6 +143,31 @@ def c2(n_seeds: int = 64, max_log_n: int = 16, max_log_b: int = 10) -> List[Work
     return [c2_pair(s, t, n_seeds, max_log_n, max_log_b) for s, t in C2_PAIRS]
 
 
+C2_ALL = ["reduce0", "reduce1", "reduce2", "reduce3", "reduce4", "reduce5", "reduce6", "reduce2_obo"]
+
+
+@dataclass
+class NWorkload:
+    """An N-kernel check (pg_check_equiv_n): kernels[k] with launch list launches[k]."""
+    name: str
+    kernels: List[str]
+    launches: List[List[Launch]]
+    n_seeds: int = 64
+    checks: int = 7
+
+
+def c2_all(n_seeds: int = 64, max_log_n: int = 16, max_log_b: int = 10) -> List[NWorkload]:
+    """SURVEY.md §8(d)'s C2 design: reduce0..reduce6 and the injected off-by-one, each
+    evaluated once per (N, B, seed), every pair compared (28 pairs).  B = 1 has no
+    reduce3..6 launch (B/2 threads), so its points form a second check of the four
+    B-thread kernels."""
+    full = c2_points(max_log_n, max_log_b, 1)
+    b1 = [(N, B) for N, B in c2_points(max_log_n, max_log_b, 0) if B == 1]
+    four = ["reduce0", "reduce1", "reduce2", "reduce2_obo"]
+    return [NWorkload("C2:all", list(C2_ALL), [[reduce_launch(k, N, B) for N, B in full] for k in C2_ALL], n_seeds),
+            NWorkload("C2:B=1", four, [[reduce_launch(k, N, B) for N, B in b1] for k in four], n_seeds)]
+
+
 # ---------------------------------------------------------------- C3
 def scan_launch(kernel: str, n: int, B: int, lognb: int = 4) -> Launch:
     sc = (n, lognb) if kernel == "prescan_padded" else (n,)

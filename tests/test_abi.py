@@ -41,16 +41,29 @@ def test_struct_sizes_match_header(pgvc):
 @pytest.mark.parametrize("bad,code", [
     ("kernel k(global out int o[4]) { o[0] = x; }", -3),
     ("kernel k(global out int o[4]) { o[0] = 1 }", -2),
-    ("kernel k(global out int o[4]) { if (tid.x == 0) { sync; } }", -3),
-    ("kernel k(global out int o[4]) { for (int i = 0; i < tid.x; i++) { sync; } }", -3),
-    ("kernel k(global out int o[4]) { while (o[0] > 0) { sync; } }", -3),
-    ("kernel k(global out int o[4]) { for (int i = 0; i < 4; i++) { if (tid.x == i) break; sync; } }", -3),
 ])
 def test_load_errors(pgvc, bad, code):
     with pytest.raises(pgvc.PgError) as e:
         pgvc.load_ir(bad)
     assert e.value.code == code
     assert re.match(r"\d+:\d+: ", str(e.value).split(": ", 1)[1])
+
+
+@pytest.mark.parametrize("text,div", [
+    ("kernel k(global out int o[4]) { if (tid.x == 0) { sync; } }", 1),
+    ("kernel k(global out int o[4]) { for (int i = 0; i < tid.x; i++) { sync; } }", 1),
+    ("kernel k(global out int o[4]) { while (o[0] > 0) { sync; } }", 1),
+    ("kernel k(global out int o[4]) { for (int i = 0; i < 4; i++) { if (tid.x == i) break; sync; } }", 1),
+    ("kernel k(global out int o[4]) { if (bdim.x > 2) { sync; } o[tid.x] = 1; }", 0),
+    ("kernel k(global out int o[4]) { for (int i = 0; i < 4; i++) { sync; } }", 0),
+])
+def test_barriers_under_thread_dependent_control_load(pgvc, text, div):
+    """X18 is checked at run time: a `sync` under thread-dependent control (tid or data) loads,
+    and is compiled with per-thread branches and resume points (PG_DIVBAR 1); block-uniform
+    barriers keep the lock-step code (PG_DIVBAR 0)."""
+    src = pgvc.load_ir(text).source()
+    assert ("#define PG_DIVBAR %d" % div) in src
+    assert "u32 sync_site(u32 k)" in src   # barrier ordinal -> site id of the BARRIER_DIV record
 
 
 def test_uniform_barriers_accepted(pgvc):
