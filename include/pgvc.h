@@ -51,6 +51,11 @@ enum { PG_IN_RAND32 = 0, PG_IN_BITS01 = 1, PG_IN_RANGE = 2 };                 /*
 enum { PG_CHK_EQUIV = 1, PG_CHK_RACE = 2, PG_CHK_OOB = 4, PG_CHK_BANK = 8, PG_CHK_COALESCE = 16,
        PG_CHK_DATAFLOW = 32, /* record the writer of every read (H5); evaluates blocks in bid order */
        PG_CHK_LOCKSTEP = 64, /* pg_check_equiv: compare the kernels' shared state round by round */
+       PG_CHK_VCLITERAL = 256, /* with PG_CHK_DATAFLOW (implied): blocks of <= 64 threads; each read's writer
+                                  is also found literally on the device - every thread s of every earlier
+                                  round tested for "s wrote the cell" (the instantiated p(s) /\ a = e(s),
+                                  L521-L522, L709-L712) - and compared with the owner-stamp writer
+                                  (pg_collect_vcliteral) */
        PG_CHK_OPCOUNT = 128  /* measurement: count the IR integer operations the kernels execute (each
                                 unary / binary / logical / select / min / max node and two per extra array
                                 dimension, under the thread's predicate) into d_counts[13]; exact
@@ -136,6 +141,21 @@ int pg_check_equiv(const pg_ir *src, const pg_ir *tgt, const pg_space *sp, pg_ru
 int pg_check_equiv_n(const pg_ir *const *ks, uint32_t nk, const pg_launch *const *launches, const pg_space *sp,
                      pg_run **out);
 
+/* Multi-kernel sequences (GKLEE's multi-kernel programs L62-L63):
+ * ks[0..n_src) is the source sequence, ks[n_src..nk) the target sequence (nk <= 8, at least
+ * one kernel each); launches[k] is phase k's launch list (n_launch points, the same parameter
+ * n; NULL = sp->launch_src).  Per (launch, seed) each side runs its phases in order on ONE
+ * set of global buffers matched by name (pair-level id, X8): a buffer starts from the PRF
+ * contents, its size is the largest any phase of the side declares, each phase checks bounds
+ * against its own declaration, and a kernel boundary is a grid-wide barrier.  Races / OOB /
+ * LIMIT / BARRIER_DIV per phase (record kernel = phase index).  The comparative assertion
+ * compares the two sides' final buffers on every id both use and some phase declares out /
+ * inout: MISMATCH in kernel 0's slot, tid fields = the last writer in the last phase of the
+ * side that declares the buffer out / inout.  Every instance runs in the exact sequential
+ * pass (blocks in bid order).  BANK / COALESCE / LOCKSTEP / DATAFLOW are PG_E_ARG. */
+int pg_check_equiv_seq(const pg_ir *const *ks, uint32_t nk, uint32_t n_src, const pg_launch *const *launches,
+                       const pg_space *sp, pg_run **out);
+
 /* Race premise of the key observation (L516-L520, L660-L662) for one kernel:
  * WW / RW / XB / OOB (and LIMIT) over the space; checks = RACE|OOB regardless
  * of sp->checks. */
@@ -190,6 +210,12 @@ int pg_collect_dataflow(pg_run *r, uint32_t *rows, size_t cap_rows, size_t *n_ro
  * Blocks of more than 1024 threads are PG_E_LIMIT in this mode; PG_E_STATE if the run
  * was not checked with PG_CHK_LOCKSTEP. */
 int pg_collect_lockstep(pg_run *r, uint32_t *rows, size_t cap_rows, size_t *n_rows);
+
+/* VC-literal cross-check of a run checked with PG_CHK_VCLITERAL:
+ * out[0] = reads whose writer was found literally, out[1] = those whose literal writer differs
+ * from the data-flow row's owner-stamp writer (0 when the ownership table is right), out[2] =
+ * literal scans that met a round beyond the 64 the history keeps.  PG_E_STATE otherwise. */
+int pg_collect_vcliteral(pg_run *r, uint64_t out[3]);
 
 /* Introspection of a loaded kernel. */
 int pg_ir_info(const pg_ir *k, uint32_t *n_sites, uint32_t *n_globals, uint32_t *n_scalars);

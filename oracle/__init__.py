@@ -80,6 +80,11 @@ def lib():
                                         ctypes.POINTER(OrRec), ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64),
                                         ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64),
                                         ctypes.POINTER(ctypes.c_uint64)]
+            _lib.or_check_seq.restype = ctypes.c_int
+            _lib.or_check_seq.argtypes = [ctypes.POINTER(ctypes.c_char_p), ctypes.c_uint32, ctypes.c_uint32,
+                                          ctypes.POINTER(ctypes.POINTER(OrLaunch)), ctypes.POINTER(OrSpace),
+                                          ctypes.POINTER(OrRec), ctypes.c_uint64, ctypes.POINTER(ctypes.c_uint64),
+                                          ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]
             _lib.or_exec.restype = ctypes.c_int
             _lib.or_exec.argtypes = [ctypes.c_char_p, ctypes.POINTER(OrLaunch), ctypes.c_uint64, ctypes.c_uint32,
                                      ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
@@ -188,6 +193,39 @@ def check_n(texts, launches, *, n_seeds=1, seed_base=0, rank=0, world=1, input_m
     counts = (ctypes.c_int64 * 16)()
     first = (ctypes.c_int64 * 11)()
     rc = L.or_check_n(tx, nk, ptrs, ctypes.byref(sp), recs, cap, ctypes.byref(n), counts, first, None)
+    if rc != 0:
+        raise OracleError(rc, L.or_last_error().decode())
+    m = min(n.value, cap)
+    out = [tuple(getattr(recs[i], f) for f in REC_FIELDS) for i in range(m)]
+    return {"records": out, "n_records": n.value, "counts": list(counts), "first_key": list(first),
+            "site_stats": None}
+
+
+def check_seq(src_texts, tgt_texts, src_launches, tgt_launches, *, n_seeds=1, seed_base=0, rank=0, world=1,
+              input_mode=0, input_range=0, bits=32, checks=EQUIV | RACE | OOB, wmax=32, cap=1 << 16):
+    """Multi-kernel sequences (or_check_seq): the source kernels run in order on one set of
+    global buffers (matched by name), so do the target kernels; final buffers compared.
+    src_launches[i] / tgt_launches[i]: launch list of phase i (same length for all).
+    Records: kernel = phase index (source phases first)."""
+    L = lib()
+    texts = list(src_texts) + list(tgt_texts)
+    launches = list(src_launches) + list(tgt_launches)
+    nk = len(texts)
+    arrs = [_launch_array(ls) for ls in launches]
+    ptrs = (ctypes.POINTER(OrLaunch) * nk)(*[ctypes.cast(a, ctypes.POINTER(OrLaunch)) for a in arrs])
+    tx = (ctypes.c_char_p * nk)(*[t.encode() for t in texts])
+    sp = OrSpace()
+    sp.launch_src = ptrs[0]
+    sp.launch_tgt = None
+    sp.n_launch = len(launches[0])
+    sp.seed_base, sp.n_seeds, sp.rank, sp.world = seed_base, n_seeds, rank, world
+    sp.input_mode, sp.input_range, sp.bits = input_mode, input_range, bits
+    sp.checks, sp.wmax, sp.mode = checks, wmax, MODE_EQUIV
+    recs = (OrRec * cap)()
+    n = ctypes.c_uint64(0)
+    counts = (ctypes.c_int64 * 16)()
+    first = (ctypes.c_int64 * 11)()
+    rc = L.or_check_seq(tx, nk, len(src_texts), ptrs, ctypes.byref(sp), recs, cap, ctypes.byref(n), counts, first)
     if rc != 0:
         raise OracleError(rc, L.or_last_error().decode())
     m = min(n.value, cap)

@@ -1179,6 +1179,10 @@ struct Exec {
     };
     std::vector<Hist> hist;
     const Hist* shadow = nullptr;   /* non-null while re-evaluating a thread of that round */
+    /* multi-kernel sequences (NEXT-4): the global buffers of the sequence so far, by pair-level
+       id; a phase starts from them (buffers a phase is the first to use: PRF contents) and
+       leaves its final contents there */
+    std::map<uint32_t, std::vector<uint32_t>>* state = nullptr;
 
     Exec(const Config& c, const KInfo& ki, const Launch& l, uint64_t sd, uint32_t li, uint32_t si, uint32_t ki_,
          Slot* sl, Results& r)
@@ -1591,7 +1595,14 @@ struct Exec {
         for (size_t a = 0; a < K.arrs.size(); a++) {
             if (K.arrs[a].space != SP_GLOBAL) continue;
             gval[a].resize(size[a]);
-            for (uint32_t i = 0; i < size[a]; i++) gval[a][i] = init_val((uint32_t)KI.gid[a], i);
+            const uint32_t g = (uint32_t)KI.gid[a];
+            if (state) {   /* sequence: the buffer as the previous phases left it */
+                std::vector<uint32_t>& b = (*state)[g];
+                for (uint32_t i = (uint32_t)b.size(); i < size[a]; i++) b.push_back(init_val(g, i));
+                for (uint32_t i = 0; i < size[a]; i++) gval[a][i] = b[i];
+            } else {
+                for (uint32_t i = 0; i < size[a]; i++) gval[a][i] = init_val(g, i);
+            }
             glast[a].assign(size[a], 0);
             gfirst_blk[a].assign(size[a], 0);
             glast_blk[a].assign(size[a], 0);
@@ -1675,6 +1686,12 @@ struct Exec {
             }
             res.instances += (uint64_t)T * cur_round;   /* X19: threads x rounds per block */
         }
+        if (state)   /* sequence: the phase's final contents stay in the buffers */
+            for (size_t a = 0; a < K.arrs.size(); a++)
+                if (K.arrs[a].space == SP_GLOBAL) {
+                    std::vector<uint32_t>& b = (*state)[(uint32_t)KI.gid[a]];
+                    for (uint32_t i = 0; i < size[a]; i++) b[i] = gval[a][i];
+                }
         /* X4: cross-block races on global cells */
         if (cfg.checks & CHK_RACE) {
             for (size_t a = 0; a < K.arrs.size(); a++) {
@@ -1751,8 +1768,11 @@ static void lockstep_compare(const Kernel& ks, uint32_t li, uint32_t sj, Results
  * global array that is out/inout in either kernel (matched by name).  A mismatch of the pair
  * is an event in slot (instance, kernel i, MISMATCH); its site field names j in N-kernel
  * checks (nmode) and is NONE for the two-kernel check. */
+static void run_seq(const std::vector<const Kernel*>& kk, const std::vector<KInfo>& ki,
+                    const std::vector<const Launch*>& lists, const Space& S, Results& res, uint32_t n_src);
+
 static void run_space(const std::vector<const Kernel*>& kk, const std::vector<const Launch*>& lists, const Space& S,
-                      Results& res, bool nmode) {
+                      Results& res, bool nmode, uint32_t seq_src = 0) {
     const int nk = (int)kk.size();
     std::vector<KInfo> ki((size_t)nk);
     /* X8: global ids = index in the sorted union of the kernels' global-array names */
@@ -1771,6 +1791,10 @@ static void run_space(const std::vector<const Kernel*>& kk, const std::vector<co
         for (size_t a = 0; a < kk[k]->arrs.size(); a++)
             if (kk[k]->arrs[a].space == SP_GLOBAL)
                 ki[k].gid[a] = (int)(std::lower_bound(names.begin(), names.end(), kk[k]->arrs[a].name) - names.begin());
+    }
+    if (seq_src) {
+        run_seq(kk, ki, lists, S, res, seq_src);
+        return;
     }
     for (uint32_t li = 0; li < S.n_launch; li++) {
         std::vector<const Launch*> LL((size_t)nk);
@@ -1823,6 +1847,65 @@ static void run_space(const std::vector<const Kernel*>& kk, const std::vector<co
     }
 }
 
+/* Multi-kernel sequences (GKLEE's multi-kernel programs L62-L63):
+ * kernels 0..n_src-1 are the source sequence, n_src.. the target sequence.  Per (launch,
+ * seed) each side runs its phases in order on ONE set of global buffers, matched by name
+ * (a kernel boundary is a grid-wide barrier: every block of phase i finishes before phase
+ * i+1 starts); a buffer's initial contents are the PRF's (X7/X8), its size the largest any
+ * phase declares, each phase checking bounds against its own declaration (X5).  Races, OOB,
+ * LIMIT, BARRIER_DIV per phase (record kernel = phase index).  The comparative assertion
+ * compares the two sides' final buffers on every name both sides use and some phase writes
+ * (out / inout): MISMATCH in kernel 0's slot, tid fields = the last writer in the side's
+ * LAST phase (NONE if that phase did not write the cell). */
+static void run_seq(const std::vector<const Kernel*>& kk, const std::vector<KInfo>& ki,
+                    const std::vector<const Launch*>& lists, const Space& S, Results& res, uint32_t n_src) {
+    const uint32_t nk = (uint32_t)kk.size();
+    for (uint32_t li = 0; li < S.n_launch; li++) {
+        for (uint32_t k = 0; k < nk; k++) check_launch(*kk[k], lists[k][li]);
+        for (uint32_t sj = S.rank; sj < S.n_seeds; sj += S.world) {
+            const uint64_t seed = S.seed_base + sj;
+            std::map<uint32_t, std::vector<uint32_t>> state[2];
+            std::map<uint32_t, std::vector<uint32_t>> last[2];   /* gid -> last writer + 1 in the side's last phase */
+            std::map<uint32_t, bool> written[2];
+            for (uint32_t k = 0; k < nk; k++) {
+                const uint32_t side = k < n_src ? 0u : 1u;
+                Slot* sl = res.slots[std::make_tuple(li, sj, k)].s;
+                Exec ex(S.cfg, ki[k], lists[k][li], seed, li, sj, k, sl, res);
+                ex.state = &state[side];
+                ex.run();
+                const bool last_phase = k == n_src - 1 || k == nk - 1;
+                for (size_t a = 0; a < kk[k]->arrs.size(); a++) {
+                    const Arr& A = kk[k]->arrs[a];
+                    if (A.space != SP_GLOBAL) continue;
+                    const uint32_t g = (uint32_t)ki[k].gid[a];
+                    if (A.mode != M_IN) written[side][g] = true;
+                    if (last_phase) last[side][g] = ex.glast[a];
+                }
+            }
+            if (!(S.cfg.checks & CHK_EQUIV)) continue;
+            Slot* sl = res.slots[std::make_tuple(li, sj, 0u)].s;
+            for (auto& kv : state[0]) {
+                const uint32_t g = kv.first;
+                if (!state[1].count(g) || !(written[0][g] || written[1][g])) continue;
+                const std::vector<uint32_t>& a = kv.second;
+                const std::vector<uint32_t>& b = state[1][g];
+                const uint32_t n = (uint32_t)std::min(a.size(), b.size());
+                for (uint32_t c = 0; c < n; c++) {
+                    if (a[c] == b[c]) continue;
+                    auto lw = [&](int side) -> uint32_t {
+                        auto it = last[side].find(g);
+                        return it != last[side].end() && c < it->second.size() ? it->second[c] - 1 : NONE32;
+                    };
+                    Ev e;
+                    uint32_t f[8] = {ROUND_END, g, c, lw(0), lw(1), NONE32, a[c], b[c]};
+                    memcpy(e.f, f, sizeof f);
+                    sl[K_MISMATCH].add(e);
+                }
+            }
+        }
+    }
+}
+
 }  // namespace orc
 
 /* ------------------------------------------------------------------ C API  */
@@ -1860,7 +1943,7 @@ const char* or_last_error(void) { return or_err.c_str(); }
  * or_check and or_check_n). */
 static int check_common(const char* const* texts, uint32_t nk, const or_launch* const* lists, bool nmode,
                         const or_space* sp, or_rec* recs, uint64_t cap, uint64_t* n_recs, int64_t* counts,
-                        int64_t* first_key, uint64_t* site_stats) {
+                        int64_t* first_key, uint64_t* site_stats, uint32_t seq_src = 0) {
     using namespace orc;
     try {
         if (!texts || !sp || !n_recs || !counts || !first_key || nk < 1 || nk > 8) throw Error(E_ARG, "null argument");
@@ -1899,7 +1982,7 @@ static int check_common(const char* const* texts, uint32_t nk, const or_launch* 
         res.max_sites = site_stats ? sp->max_sites : 0;
         res.stats_nk = std::max<uint32_t>(2, nk);
         res.site_stats.assign((size_t)sp->n_launch * res.stats_nk * res.max_sites * 8, 0);
-        run_space(kk, ll, S, res, nmode);
+        run_space(kk, ll, S, res, nmode, seq_src);
         for (int i = 0; i < 16; i++) counts[i] = 0;
         for (int i = 0; i < 11; i++) first_key[i] = INT64_MAX;
         counts[0] = (int64_t)res.instances;
@@ -1963,6 +2046,18 @@ int or_check_n(const char* const* texts, uint32_t nk, const or_launch* const* la
                or_rec* recs, uint64_t cap, uint64_t* n_recs, int64_t* counts, int64_t* first_key,
                uint64_t* site_stats) {
     return check_common(texts, nk, launches, true, sp, recs, cap, n_recs, counts, first_key, site_stats);
+}
+
+/* Multi-kernel sequences: texts[0..n_src) the source sequence, texts[n_src..nk) the target
+ * sequence (run_seq).  n_src >= 1, nk - n_src >= 1, nk <= 8. */
+int or_check_seq(const char* const* texts, uint32_t nk, uint32_t n_src, const or_launch* const* launches,
+                 const or_space* sp, or_rec* recs, uint64_t cap, uint64_t* n_recs, int64_t* counts,
+                 int64_t* first_key) {
+    if (n_src < 1 || n_src >= nk) {
+        or_err = "a sequence check needs at least one kernel on each side";
+        return -1;
+    }
+    return check_common(texts, nk, launches, false, sp, recs, cap, n_recs, counts, first_key, nullptr, n_src);
 }
 
 /* Run one kernel for one launch/seed and return its initial and final global

@@ -743,6 +743,7 @@ struct Gen {
         o << "#define PG_FAST " << (O.fast ? 1 : 0) << "\n";
         o << "#define PG_DIVBAR " << (K.div_barrier ? 1 : 0) << "\n";
         o << "#define PG_OPCOUNT " << ((O.checks & 128) ? 1 : 0) << "\n";
+        o << "#define PG_VCLIT " << ((O.checks & 256) ? 1 : 0) << "\n";
         o << "#define PG_WMAX " << O.wmax << "\n";
         o << "#define PG_MS " << (ms() ? O.ms : 1u) << "\n";
         o << "#define PG_NSTATS " << std::max<size_t>(1, K.sites.size()) << "\n";

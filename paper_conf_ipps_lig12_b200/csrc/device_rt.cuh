@@ -397,8 +397,56 @@ struct PgDf {
     u32 cap;
 };
 __shared__ PgDf pg_sDf;  // data-flow recorder of this CTA
+#ifndef PG_VCLIT
+#define PG_VCLIT 0
+#endif
+#define PG_HIST_R 64u   // rounds per block the VC-literal history keeps
+#if PG_VCLIT
+// GPU VC-literal mode: the
+// writer of a read found by enumerating, for every earlier round (latest first; shared cells:
+// this block's rounds, global cells: every block run so far, in bid order), every thread s
+// of that round and testing "s wrote the cell" on s's logged writes of the round - the
+// instantiated p(s) ∧ a = e(s) - instead of the owner stamps.  It must equal the data-flow
+// row's owner-stamp writer (min s under WW); disagreements are counted (header word 1).
+__device__ __noinline__ void pg_vclit(const PgC& C, const PgT& t, u32 cell, u32 glob, u32 src, u32 wb, u32 wr,
+                                      u32 wg) {
+    const u32 T = PG_T, HW = 1u + (u32)PG_WMAX;
+    const u32* hist = t.arena + pg_sL.off_hist;
+    const u32* hr = t.arena + pg_sL.off_hround;
+    u32 fb = PG_NEVER, fr = PG_NEVER, fs = PG_NEVER;
+    for (int b = (int)t.blk; b >= 0 && fs == PG_NEVER; b--) {
+        if (!glob && (u32)b != t.blk) break;
+        const u32 nr = (u32)b == t.blk ? C.round : hr[b];
+        for (int r = (int)nr - 1; r >= 0 && fs == PG_NEVER; r--) {
+            if ((u32)r >= PG_HIST_R) {   // (a round the history does not keep)
+                atomicAdd(pg_sDf.count + 2, 1u);
+                continue;
+            }
+            for (u32 s = 0; s < T; s++) {
+                const u32* e = hist + (((u64)b * PG_HIST_R + (u32)r) * T + s) * HW;
+                const u32 n = min(e[0], (u32)PG_WMAX);
+                for (u32 i = 0; i < n; i++)
+                    if (e[1 + i] == cell) {
+                        fs = min(fs, s);
+                        break;
+                    }
+            }
+            if (fs != PG_NEVER) {
+                fb = (u32)b;
+                fr = (u32)r;
+            }
+        }
+    }
+    const bool ok = src == 0u ? fs == PG_NEVER : (fb == wb && fr == wr && fb * T + fs == wg);
+    atomicAdd(pg_sDf.count + 3, 1u);
+    if (!ok) atomicAdd(pg_sDf.count + 1, 1u);
+}
+#endif
 __device__ __noinline__ void pg_df_row(const PgC& C, const PgT& t, u32 site, u32 rec, u32 flat, u32 src, u32 wb, u32 wr,
-                                       u32 wg) {
+                                       u32 wg, u32 cell, u32 glob) {
+#if PG_VCLIT
+    if (src != 2u) pg_vclit(C, t, cell, glob, src, wb, wr, wg);
+#endif
     const u32 i = atomicAdd(pg_sDf.count, 1u);
     if (i >= pg_sDf.cap) return;
     u32* r = pg_sDf.rows + (u64)i * 12u;
@@ -409,11 +457,11 @@ __device__ __noinline__ void pg_df_row(const PgC& C, const PgT& t, u32 site, u32
 }
 // writer of a committed global cell: last committer (gtid) and the round of its stamp
 __device__ __forceinline__ void pg_df_global(const PgC& C, const PgT& t, u32 site, u32 rec, u32 flat, u32 lw, u32 own,
-                                             u64 off_step0) {
-    if (!lw) { pg_df_row(C, t, site, rec, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER); return; }
+                                             u64 off_step0, u32 cell) {
+    if (!lw) { pg_df_row(C, t, site, rec, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER, cell, 1u); return; }
     const u32 wg = lw - 1u, wb = wg / PG_T;
     const u32 s0 = wb == t.blk ? C.step0 : t.arena[off_step0 + wb];
-    pg_df_row(C, t, site, rec, flat, 1u, wb, pg_owner_step(own) - s0, wg);
+    pg_df_row(C, t, site, rec, flat, 1u, wb, pg_owner_step(own) - s0, wg, cell, 1u);
 }
 #endif
 
@@ -483,7 +531,7 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
     u32 v;
     if (LOG && pg_log_find(t, c, ((u32)A << 24) | flat, v)) {
 #if PG_DATAFLOW
-        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 2u, t.blk, C.round, t.gtid);
+        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 2u, t.blk, C.round, t.gtid, ((u32)A << 24) | flat, 0u);
 #endif
         return v;
     }
@@ -494,13 +542,13 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
         PG_EVENT(t, c, PGK_UNINIT, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, pv, 0);
 #endif
 #if PG_DATAFLOW
-        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER);
+        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER, ((u32)A << 24) | flat, 0u);
 #endif
         return pv;
     }
 #if PG_DATAFLOW
     pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 1u, t.blk, pg_owner_step(own) - C.step0,
-              t.blk * PG_T + (own & 0xFFFu));
+              t.blk * PG_T + (own & 0xFFFu), ((u32)A << 24) | flat, 0u);
 #endif
     return pg_sh(t, PG_SH(A, s_val))[flat];
 }
@@ -1057,13 +1105,13 @@ __device__ __forceinline__ u32 pg_ld_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
     u32 v;
     if (LOG && pg_log_find(t, c, ((u32)A << 24) | flat, v)) {
 #if PG_DATAFLOW
-        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 2u, t.blk, C.round, t.gtid);
+        pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 2u, t.blk, C.round, t.gtid, ((u32)A << 24) | flat, 1u);
 #endif
         return v;
     }
 #if PG_DATAFLOW
     pg_df_global(C, t, site, PG_ARR(A).rec_id, flat, t.arena[PG_ARR(A).off_lw + flat],
-                 t.arena[PG_ARR(A).off_own + flat], pg_sL.off_step0);
+                 t.arena[PG_ARR(A).off_own + flat], pg_sL.off_step0, ((u32)A << 24) | flat);
 #endif
     return t.arena[PG_ARR(A).off_val + flat];
 #endif
@@ -1119,7 +1167,7 @@ __device__ __forceinline__ u32 pg_ld_gi(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
         return pv;
     }
 #if PG_DATAFLOW
-    pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER);
+    pg_df_row(C, t, site, PG_ARR(A).rec_id, flat, 0u, PG_NEVER, PG_NEVER, PG_NEVER, ((u32)A << 24) | flat, 1u);
 #endif
     return __ldg(t.input + PG_ARR(A).off_in + flat);
 }
@@ -1232,6 +1280,18 @@ __device__ __forceinline__ void pg_check_gt(const PgC& C, PgT& t, PgCold& c, u32
 #endif
 }
 
+#if PG_VCLIT
+// VC-literal history: this thread's logged writes of the round (every real thread writes its
+// count, 0 when it wrote nothing or has exited)
+__device__ __forceinline__ void pg_hist_put(const PgC& C, const PgT& t, const PgCold& c) {
+    if (t.ekey == 63u || t.blk >= pg_sW.blk1 || C.round >= PG_HIST_R) return;
+    u32* e = t.arena + pg_sL.off_hist + (((u64)t.blk * PG_HIST_R + C.round) * PG_T + t.tlin) * (1u + (u32)PG_WMAX);
+    e[0] = t.nlog;
+    if (t.nlog) e[1] = t.l0cell;
+    for (u32 i = 1; i < t.nlog; i++) e[1 + i] = c.lcell[i];
+}
+#endif
+
 template <class K>
 __device__ __forceinline__ void pg_claim_all(const PgC& C, const PgT& t, const PgCold& c) {
     // a 1-thread block is the only writer of its cells in the round (other blocks sharing a
@@ -1315,6 +1375,9 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
     pg_claim_all<K>(C, t, c);
     if (warp_blocks) __syncwarp(); else __syncthreads();
     pg_check_all<K>(C, t, c);
+#if PG_VCLIT
+    pg_hist_put(C, t, c);
+#endif
 #if PG_LOCKSTEP
     if (warp_blocks) __syncwarp(); else __syncthreads();
     pg_snapshot(C, t);
@@ -1665,7 +1728,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 const PgArr& R = pg_sL.arr[a];
                 if (R.kind != PGA_GT) continue;
                 for (u32 i = threadIdx.x; i < R.size; i += blockDim.x) {
-                    ar[R.off_val + i] = pg_init_value(P, seed, R.gid, i);
+                    if (!P.keep_vals) ar[R.off_val + i] = pg_init_value(P, seed, R.gid, i);
                     ar[R.off_own + i] = PG_NEVER;
                     ar[R.off_lw + i] = 0u;
                     if (R.off_wmax != ~0ull) ar[R.off_wmax + i] = 0u;
@@ -1817,6 +1880,9 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             t.fuel = 0;
             alive_rounds = t.live;
             K::run(F[0], C, t, Cd[0], sstats, alive_rounds);
+#if PG_VCLIT
+            if (inst_ok && tl0 == 0u && blk_ok) t.arena[pg_sL.off_hround + blk] = C.round;
+#endif
         }
 #else
         u32 resume = 0;

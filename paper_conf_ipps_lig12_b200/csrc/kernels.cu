@@ -148,8 +148,8 @@ __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs
     }
 }
 
-__device__ __forceinline__ u32 pg_cmp_lw(const PgRegions& R, u32 r, u64 lw, u64 inst, u64 stride, u32 addr) {
-    return r == PG_R_INPUT ? PG_NEVER : R.r[r][lw + inst * stride + addr] - 1u;
+__device__ __forceinline__ u32 pg_cmp_lw(const PgRegions& R, u32 r, u32 has, u64 lw, u64 inst, u64 stride, u32 addr) {
+    return has ? R.r[r][lw + inst * stride + addr] - 1u : PG_NEVER;
 }
 
 // K3b: among the pairs (i, j) that mismatch at kernel i's minimum cell, the minimum
@@ -167,7 +167,7 @@ __global__ void __launch_bounds__(128) pg_compare_pick(const PgCmp* __restrict__
     const u32 a = R.r[c.src_r][c.src_off + (u64)inst * c.src_stride + addr];
     const u32 b = R.r[c.tgt_r][c.tgt_off + (u64)inst * c.tgt_stride + addr];
     if (a == b) return;
-    const u32 tb = pg_cmp_lw(R, c.tgt_r, c.tgt_lw, inst, c.tgt_stride, addr);
+    const u32 tb = pg_cmp_lw(R, c.tgt_r, c.lw_flags & 2u, c.tgt_lw, inst, c.tgt_stride, addr);
     atomicMin(&mm2[mi], ((u64)tb << 32) | c.site);
 }
 
@@ -185,13 +185,13 @@ __global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__
     if (addr >= c.n) return;
     const u32 a = R.r[c.src_r][c.src_off + (u64)inst * c.src_stride + addr];
     const u32 b = R.r[c.tgt_r][c.tgt_off + (u64)inst * c.tgt_stride + addr];
-    const u32 tb = pg_cmp_lw(R, c.tgt_r, c.tgt_lw, inst, c.tgt_stride, addr);
+    const u32 tb = pg_cmp_lw(R, c.tgt_r, c.lw_flags & 2u, c.tgt_lw, inst, c.tgt_stride, addr);
     if (a == b || mm2[mi] != (((u64)tb << 32) | c.site)) return;
     PgSlot* s = &slots[c.slot0 + (u64)inst * c.slot_step];
     s->f[0] = 0xFFFFu;
     s->f[1] = c.gid;
     s->f[2] = addr;
-    s->f[3] = pg_cmp_lw(R, c.src_r, c.src_lw, inst, c.src_stride, addr);
+    s->f[3] = pg_cmp_lw(R, c.src_r, c.lw_flags & 1u, c.src_lw, inst, c.src_stride, addr);
     s->f[4] = tb;
     s->f[5] = c.site;
     s->f[6] = a;

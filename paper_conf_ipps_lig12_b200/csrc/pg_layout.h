@@ -59,6 +59,8 @@ struct PgLaunchK {
     u32 smem_group_bytes, smem_zero_off, smem_never_off, n_arrays;
     u64 arena_stride, input_stride;          // u32 words per instance
     u64 off_step0;                           // data-flow mode: per-block first round step (arena words), ~0 absent
+    u64 off_hist, off_hround;                // VC-literal mode: [block][round < 64][thread][1 + W_max] logged
+                                             // writes, [block] rounds (arena words), ~0 absent
     PgArr arr[PG_MAXARR];
 };
 
@@ -115,6 +117,9 @@ struct PgParams {
     u32* flag_any;          // set when any instance of the batch is flagged; re-run passes with
                             // nothing flagged exit at once (nullptr: absent)
     u64* op_cnt;            // PG_CHK_OPCOUNT: per batch-local instance, IR integer operations executed
+    u32 keep_vals;          // sequential pass of a later phase of a kernel sequence: the global values
+                            // are the previous phase's results (only stamps are reset)
+    u32 pad4;
 };
 
 // K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive
@@ -179,4 +184,6 @@ struct PgCmp {
     u32 task0;                   // first CTA task (pg_fill_tasks(n, n_inst))
     u32 site;                    // record site field: j in N-kernel checks, PG_NEVER for a pair
     u64 mm0, mm_step;            // per-(instance, kernel i) minimum-cell words of instance 0, stride
+    u32 lw_flags;                // bit 0 / 1: the source / target side has last-writer words (else NONE)
+    u32 pad;
 };

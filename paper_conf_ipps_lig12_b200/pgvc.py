@@ -18,6 +18,7 @@ LIB_PATH = os.path.join(_HERE, "libpgvc.so")
 PG_OK, PG_E_ARG, PG_E_PARSE, PG_E_TYPE, PG_E_LIMIT, PG_E_CUDA, PG_E_OOM, PG_E_STATE = 0, -1, -2, -3, -4, -5, -6, -7
 IN_RAND32, IN_BITS01, IN_RANGE = 0, 1, 2
 CHK_EQUIV, CHK_RACE, CHK_OOB, CHK_BANK, CHK_COALESCE, CHK_DATAFLOW, CHK_LOCKSTEP, CHK_OPCOUNT = 1, 2, 4, 8, 16, 32, 64, 128
+CHK_VCLITERAL = 256
 LOCK_ROUNDS = 32
 BANKS_32, BANKS_16_HALFWARP = 0, 1
 KINDS = ["BARRIER_DIV", "OOB", "RACE_WW", "RACE_RW", "RACE_XB", "MISMATCH", "BANK", "UNCOALESCED", "UNINIT", "LIMIT"]
@@ -74,8 +75,9 @@ class PgError(RuntimeError):
 
 
 _lib = None
-EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
-           "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info", "pg_ir_seed_oblivious",
+EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_equiv_seq", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
+           "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_collect_vcliteral", "pg_ir_info",
+           "pg_ir_seed_oblivious",
            "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals", "pg_merge_counters",
            "pg_measure_int32_peak",
            "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
@@ -96,6 +98,9 @@ def lib():
     L.pg_check_races.argtypes = [vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_check_equiv_n.argtypes = [ctypes.POINTER(vp), ctypes.c_uint32, ctypes.POINTER(ctypes.POINTER(PgLaunch)),
                                    ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
+    L.pg_check_equiv_seq.argtypes = [ctypes.POINTER(vp), ctypes.c_uint32, ctypes.c_uint32,
+                                     ctypes.POINTER(ctypes.POINTER(PgLaunch)), ctypes.POINTER(PgSpace),
+                                     ctypes.POINTER(vp)]
     L.pg_check_banks.argtypes = [vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_check_property.argtypes = [vp, vp, ctypes.POINTER(PgSpace), ctypes.POINTER(vp)]
     L.pg_collect_cex.argtypes = [vp, ctypes.POINTER(PgCex), ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t),
@@ -105,6 +110,7 @@ def lib():
                                       ctypes.POINTER(ctypes.c_size_t)]
     L.pg_collect_dataflow.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.c_size_t,
                                       ctypes.POINTER(ctypes.c_size_t)]
+    L.pg_collect_vcliteral.argtypes = [vp, ctypes.POINTER(ctypes.c_uint64)]
     L.pg_ir_info.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32),
                              ctypes.POINTER(ctypes.c_uint32)]
     L.pg_ir_seed_oblivious.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32)]
@@ -121,8 +127,9 @@ def lib():
     L.pg_version.restype = ctypes.c_char_p
     L.pg_ir_free.argtypes = [vp]
     L.pg_run_free.argtypes = [vp]
-    for f in ("pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
-              "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_ir_info",
+    for f in ("pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_equiv_seq", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
+              "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_collect_vcliteral",
+              "pg_ir_info",
               "pg_ir_seed_oblivious", "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals",
               "pg_merge_counters", "pg_measure_int32_peak"):
         getattr(L, f).restype = ctypes.c_int
@@ -297,6 +304,13 @@ class Run:
         out = out[:min(n.value, 1 << 20)]
         return out[np.lexsort(out.T[::-1])] if len(out) else out
 
+    def vcliteral(self):
+        """(reads checked literally, disagreements with the owner-stamp writer, history
+        overflows) of a CHK_VCLITERAL run (pg_collect_vcliteral)."""
+        out = (ctypes.c_uint64 * 3)()
+        _ck(lib().pg_collect_vcliteral(self._h, out))
+        return {"checked": out[0], "disagree": out[1], "overflow": out[2]}
+
     def lockstep(self):
         """First shared-state divergence per instance of a PG_CHK_LOCKSTEP equivalence run:
         list of tuples in LOCK_FIELDS order, (launch, seed) order."""
@@ -339,6 +353,42 @@ def _run(fn, irs, space: Space) -> Run:
 
 def pg_check_equiv(src: Ir, tgt: Ir, space: Space) -> Run:
     return _run(lib().pg_check_equiv, [src, tgt], space)
+
+
+def _launch_ptrs(space: Space, launches, tag: str):
+    n = len(launches[0])
+    if any(len(l) != n for l in launches):
+        raise PgError(PG_E_ARG, "launch lists of different lengths")
+    key = (id(launches), len(launches), n)
+    cached = space.__dict__.get(tag)   # (marshalled once per Space object, as marshal() does)
+    if cached is not None and cached[0] == key:
+        return n, cached[1], cached[2]
+    arrs = [(PgLaunch * max(1, n))(*[_launch(l) for l in ls]) for ls in launches]
+    ptrs = (ctypes.POINTER(PgLaunch) * len(arrs))(*[ctypes.cast(a, ctypes.POINTER(PgLaunch)) for a in arrs])
+    space.__dict__[tag] = (key, arrs, ptrs)
+    return n, arrs, ptrs
+
+
+def pg_check_equiv_seq(src: Sequence[Ir], tgt: Sequence[Ir], src_launches: Sequence[Sequence],
+                       tgt_launches: Sequence[Sequence], space: Space) -> Run:
+    """Kernel sequences (pg_check_equiv_seq): the source kernels run in order on one set of
+    global buffers, so do the target kernels; final buffers compared.  *_launches[i] is
+    phase i's launch list."""
+    kernels = list(src) + list(tgt)
+    if len(src) < 1 or len(tgt) < 1 or len(kernels) > 8:
+        raise PgError(PG_E_ARG, "1 to 7 kernels per side, 8 in all")
+    launches = list(src_launches) + list(tgt_launches)
+    if len(launches) != len(kernels):
+        raise PgError(PG_E_ARG, "one launch list per kernel")
+    sp, keep = space.marshal()
+    n, arrs, ptrs = _launch_ptrs(space, launches, "_seq_arrays")
+    sp.launch_src = ptrs[0]
+    sp.launch_tgt = None
+    sp.n_launch = n
+    hs = (ctypes.c_void_p * len(kernels))(*[k.handle.value for k in kernels])
+    h = ctypes.c_void_p()
+    _ck(lib().pg_check_equiv_seq(hs, len(kernels), len(src), ptrs, ctypes.byref(sp), ctypes.byref(h)))
+    return Run(h, space, (keep, arrs, ptrs, kernels))
 
 
 def pg_check_equiv_n(kernels: Sequence[Ir], launches: Sequence[Sequence], space: Space) -> Run:
@@ -384,7 +434,7 @@ def pg_check_property(k: Ir, post: Ir, space: Space) -> Run:
 
 
 check_equiv, check_races, check_banks, check_property = pg_check_equiv, pg_check_races, pg_check_banks, pg_check_property
-check_equiv_n = pg_check_equiv_n
+check_equiv_n, check_equiv_seq = pg_check_equiv_n, pg_check_equiv_seq
 
 
 def merge_counters(first_keys, counts, out_first_key, out_counts, stream: int = 0):

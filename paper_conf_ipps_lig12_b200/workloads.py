@@ -256,3 +256,29 @@ def scalar_prod_launch(vectorN: int, elementN: int, accn: int, bdim: int) -> Lau
 def accn_sweep(max_accn: int = 16, bdims=(1, 4, 8), vectorN: int = 2, elementN: int = 40) -> List[Launch]:
     """ACCN = 1..max_accn in order (the witness order), for each block size."""
     return [scalar_prod_launch(vectorN, elementN, a, b) for a in range(1, max_accn + 1) for b in bdims]
+
+
+@dataclass
+class SeqWorkload:
+    """A sequence check (pg_check_equiv_seq): the source kernels run in order on one set of
+    global buffers, so do the target kernels; launches[i] is phase i's launch list."""
+    name: str
+    src: List[str]
+    tgt: List[str]
+    src_launches: List[List[Launch]]
+    tgt_launches: List[List[Launch]]
+    n_seeds: int = 64
+    checks: int = 7
+
+
+def reduce_two_pass(n_seeds: int = 8, max_log_n: int = 14, max_log_b: int = 10, first: str = "reduce0",
+                    second: str = "reduce0_pass2") -> SeqWorkload:
+    """The SDK's multi-pass reduction as a kernel sequence (GKLEE multi-kernel programs,
+    PAPER.md L62-L63): `first` reduces N inputs to M = N/B block sums (g_odata), `second`
+    reduces those in one block of M threads into g_sum[0]; the target is the one-thread
+    specification sum_serial.  Points (N, B) with M = N/B <= 1024, powers of two."""
+    pts = [(N, B) for N, B in c2_points(max_log_n, max_log_b, 0) if N // B <= 1024]
+    p1 = [reduce_launch(first, N, B) for N, B in pts]
+    p2 = [Launch((1, 1, 1), (N // B, 1, 1), (N // B,)) for N, B in pts]
+    ser = [Launch((1, 1, 1), (1, 1, 1), (N,)) for N, B in pts]
+    return SeqWorkload("C2:two-pass", [first, second], ["sum_serial"], [p1, p2], [ser], n_seeds)
