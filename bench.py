@@ -1,13 +1,17 @@
-"""pgvc benchmark — VC instances checked per second (BASELINE.json metric).
+"""pgvc benchmark - VC instances checked per second (BASELINE.json metric).
 
-Workload (N=1 headline, BASELINE.json configs[1] = C2): CUDA SDK reduction variants
-reduce0..reduce6 checked pairwise against reduce0 plus the injected off-by-one pair
-(reduce2 vs reduce2_obo); B = 2^0..2^10 elements per block, N = B..2^16, 64 seeds
-per GPU (RAND32), checks EQUIV|RACE|OOB.  One step = every pair over the whole
-space: input generation (K1), both evaluation kernels (K2), comparison (K3),
-compaction (K4) and the H9 all_reduce of the first-counterexample key (MIN) and
-the counts (SUM).  Multi-GPU: N ranks shard a 64 x N seed space round-robin
-(64 seeds per GPU, weak scaling); the only collective is H9.
+Workload (N=1 headline, BASELINE.json configs[1] = C2, in SURVEY.md §8(d)'s design):
+the CUDA SDK reduction variants reduce0..reduce6 and the injected off-by-one reduce2_obo,
+each evaluated ONCE per (N, B, seed) and every pair compared (pg_check_equiv_n; 28 pairs,
+the 21 of reduce0..6 among them); B = 2^1..2^10 elements per block, N = B..2^16, plus the
+B = 1 points as a 4-kernel check (reduce3..6 have no B/2 = 0 thread launch); 64 seeds per
+GPU (RAND32), checks EQUIV|RACE|OOB.  One step = both checks over the whole space: input
+generation (K1), the evaluation kernels (K2), comparison (K3), compaction (K4), the
+device-side merge of the checks' counters (K5) and the H9 all_reduce of the first-
+counterexample key (MIN) and the counts (SUM).  `--workload c2` runs C2 as seven pairs
+(reduce0 against reduce1..6, reduce2 against reduce2_obo; round 1's design).  Multi-GPU: N
+ranks shard a 64 x N seed space round-robin (64 seeds per GPU, weak scaling); the only
+collective is H9.
 
 `--impl reference` times the CPU oracle (oracle/, test infrastructure) on the
 host cores on a bounded sample of the same workload.
@@ -59,7 +63,7 @@ WORKLOADS = {
     "c5m": ("C5 matmul: naive vs 32x32 tiled, N = 32..1024, K = 64, %d seeds per GPU", 1250, (650 + 678) // 6,
             lambda W, s: [W.c5_matmul(n_seeds=s)]),
 }
-WL = "c2"
+WL = "c2n"
 
 
 def workload_desc():
@@ -262,8 +266,9 @@ def main():
     ap.add_argument("--ref-seeds", type=int, default=SAMPLE_SEEDS, help="oracle sample: seeds 0..k-1")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + 1 step, no JSON (for ncu launch lists)")
     ap.add_argument("--diag", action="store_true", help="print per-step enqueue / device / per-check times")
-    ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS),
-                    help="c2 (headline, BASELINE configs[1]); others: the remaining configs for reference")
+    ap.add_argument("--workload", default="c2n", choices=sorted(WORKLOADS),
+                    help="c2n (headline, BASELINE configs[1] in the survey's design); c2: the same space as seven "
+                         "pairs; others: the remaining configs")
     ap.add_argument("--streams", type=int, default=0,
                     help="streams the independent pairs are spread over (default 0: one per pair; 1: one stream)")
     ap.add_argument("--seeds", type=int, default=0, help="seeds per GPU (default: the workload's)")

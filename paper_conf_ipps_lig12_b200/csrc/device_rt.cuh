@@ -186,8 +186,12 @@ struct PgCold {     // per-emulated-thread state that lives in local memory
     u32 ebest[PG_NK][8];  // minimum event per kind  so threads without events touch no local memory) (X16)
 #if PG_MSX
     u32 lvs[PG_WMAX][PG_MS];   // (see pg_lv_t)     // write-log values per seed (entries 1..)
-    u32 ebv[PG_NK][PG_MS][2];    // per seed: (val_a, val_b) of the minimum event; fields 0..5 of
-                                 // ebest are seed-independent (same accesses in every seed)
+    u32 ebv[PG_NK][PG_MS];       // per seed: val_a of the minimum event; fields 0..5 of ebest are
+                                 // seed-independent (same accesses in every seed)
+    u32 ebvb[PG_NK];             // its val_b, which every event kind takes seed-independently (site,
+                                 // degree, ...), so one word per kind (local-memory footprint) ...
+    u32 vbx;                     // ... unless two events with equal fields 0..5 but different val_b
+    u32 ebvs[PG_NK][PG_MS];      //     met (bit k): then val_b per seed here
     u64 epk[PG_NK];              // pg_pack of ebest[kind] (one 64-bit compare decides most events)
 #endif
 };
@@ -801,15 +805,24 @@ __device__ __noinline__ u32 pg_event_ms(PgCold& c, u32 evm, u32 kind, u32 round,
         for (int i = 0; i < 6 && cmp == 0; i++)
             if (e[i] != c.ebest[kind][i]) cmp = e[i] < c.ebest[kind][i] ? -1 : 1;
     }
+    const u32 nvx = evm ? c.vbx : 0u;   // (the thread's first event initialises vbx)
     if (cmp < 0) {
         c.epk[kind] = pk;
         for (int i = 0; i < 6; i++) c.ebest[kind][i] = e[i];
-        PG_S_LOOP { c.ebv[kind][_s][0] = va[_s]; c.ebv[kind][_s][1] = vb; }
+        PG_S_LOOP c.ebv[kind][_s] = va[_s];
+        c.ebvb[kind] = vb;
+        c.vbx = nvx & ~(1u << kind);
     } else if (cmp == 0) {   // same access: the per-seed values decide (X16 lexicographic order)
-        PG_S_LOOP {
-            if (va[_s] < c.ebv[kind][_s][0] || (va[_s] == c.ebv[kind][_s][0] && vb < c.ebv[kind][_s][1])) {
-                c.ebv[kind][_s][0] = va[_s];
-                c.ebv[kind][_s][1] = vb;
+        if (!((nvx >> kind) & 1u) && vb == c.ebvb[kind]) {
+            PG_S_LOOP if (va[_s] < c.ebv[kind][_s]) c.ebv[kind][_s] = va[_s];
+        } else {   // (rare: val_b may now differ between seeds)
+            if (!((nvx >> kind) & 1u)) PG_S_LOOP c.ebvs[kind][_s] = c.ebvb[kind];
+            c.vbx = nvx | (1u << kind);
+            PG_S_LOOP {
+                if (va[_s] < c.ebv[kind][_s] || (va[_s] == c.ebv[kind][_s] && vb < c.ebvs[kind][_s])) {
+                    c.ebv[kind][_s] = va[_s];
+                    c.ebvs[kind][_s] = vb;
+                }
             }
         }
     }
@@ -1471,8 +1484,8 @@ __device__ __noinline__ void pg_flush_cta(const PgParams& P, u32 lane, u32 warp,
 #pragma unroll
             for (int i = 0; i < 8; i++) f_in[i] = pending ? c.ebest[k][i] : PG_NEVER;
 #if PG_MSX
-            f_in[6] = pending ? c.ebv[k][seed_s][0] : PG_NEVER;   // (multi-seed exact pass: this seed's values)
-            f_in[7] = pending ? c.ebv[k][seed_s][1] : PG_NEVER;
+            f_in[6] = pending ? c.ebv[k][seed_s] : PG_NEVER;   // (multi-seed exact pass: this seed's values)
+            f_in[7] = pending ? ((c.vbx >> k) & 1u ? c.ebvs[k][seed_s] : c.ebvb[k]) : PG_NEVER;
 #endif
             pg_warp_merge(pending, slot0, pending ? c.ecnt[k] : 0u, f_in, lane, leader, key, cnt, best, members);
             if (lane == leader) {
@@ -1581,8 +1594,8 @@ __device__ __noinline__ void pg_flush_cta_ms(const PgParams& P, u32 lane, u32 wa
             u32 vv[PG_MS][2];
 #pragma unroll
             for (u32 q = 0; q < PG_MS; q++) {
-                vv[q][0] = __shfl_sync(PG_FULL, c.ebv[k][q][0], win);
-                vv[q][1] = __shfl_sync(PG_FULL, c.ebv[k][q][1], win);
+                vv[q][0] = __shfl_sync(PG_FULL, c.ebv[k][q], win);
+                vv[q][1] = __shfl_sync(PG_FULL, (c.vbx >> k) & 1u ? c.ebvs[k][q] : c.ebvb[k], win);
             }
             const u32 wn = __shfl_sync(PG_FULL, nsv, win);
             if (lane == leader) {

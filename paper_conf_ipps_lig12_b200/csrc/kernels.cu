@@ -97,106 +97,160 @@ __global__ void __launch_bounds__(256) pg_gen_inputs(const PgFill* __restrict__ 
     }
 }
 
-// K3a: count mismatching cells per (instance, pair, array); keep the minimum (gid, addr) per
-// (instance, kernel i) - the pairs (i, j) of an N-kernel check share kernel i's MISMATCH slot.
-// One CTA task per grid-stride step (pg_task_job).
+// K3a: per (instance, array) job cell by cell: every member's value once; for each member a
+// the mismatching pairs (a, b > a) - their count into kernel kid[a]'s MISMATCH slot and the
+// minimum mismatching cell into its (instance, kernel) word.  One CTA task per grid-stride
+// step (pg_task_job).
+__device__ __forceinline__ bool pg_pair(const PgCmp& c, u32 a, u32 b, u32 i) {
+    return ((c.pair_mask >> (a * PG_MAXK + b)) & 1ull) && i < c.size[a] && i < c.size[b];
+}
+// the members' value rows of one instance, with their sizes (registers for the cell loop)
+struct PgCmpRows {
+    const u32* p[PG_MAXK];
+    u32 size[PG_MAXK];
+    u64 mask;
+    u32 nm;
+};
+__device__ __forceinline__ void pg_cmp_rows(const PgCmp& c, const PgRegions& R, u32 inst, PgCmpRows& w) {
+    w.nm = c.nm;
+    w.mask = c.pair_mask;
+#pragma unroll
+    for (u32 m = 0; m < PG_MAXK; m++) {
+        const bool on = m < c.nm;
+        w.p[m] = on ? R.r[c.region[m]] + c.off[m] + (u64)inst * c.stride[m] : nullptr;
+        w.size[m] = on ? c.size[m] : 0u;
+    }
+}
+__device__ __forceinline__ void pg_cmp_cell(const PgCmpRows& w, u32 i, u32 (&cnt)[PG_MAXK], u32 (&mn)[PG_MAXK]) {
+    u32 v[PG_MAXK];
+#pragma unroll
+    for (u32 m = 0; m < PG_MAXK; m++) v[m] = i < w.size[m] ? w.p[m][i] : 0u;
+#pragma unroll
+    for (u32 a = 0; a + 1 < PG_MAXK; a++) {
+        u32 k = 0;
+#pragma unroll
+        for (u32 b = a + 1; b < PG_MAXK; b++)
+            k += (v[a] != v[b]) & (u32)((w.mask >> (a * PG_MAXK + b)) & 1ull) & (i < w.size[a]) & (i < w.size[b]);
+        if (k) {
+            cnt[a] += k;
+            mn[a] = min(mn[a], i);
+        }
+    }
+}
 __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs, u32 n_jobs, u32 n_tasks,
                                                   const PgRegions R, PgSlot* slots, u64* mm_key) {
-    __shared__ u32 s_cnt;
-    __shared__ u32 s_min;
+    __shared__ u32 s_cnt[PG_MAXK], s_min[PG_MAXK];
     __shared__ u32 s_job;
     if (threadIdx.x == 0) s_job = 0u;
     for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
-        const PgCmp c = jobs[pg_task_job(jobs, n_jobs, 0u, task, &s_job)];
+        const PgCmp& c = jobs[pg_task_job(jobs, n_jobs, 0u, task, &s_job)];
         const u32 lt = task - c.task0;
-        const u32* rs = R.r[c.src_r];
-        const u32* rt = R.r[c.tgt_r];
+        u32 cnt[PG_MAXK], mn[PG_MAXK];
+#pragma unroll
+        for (u32 m = 0; m < PG_MAXK; m++) { cnt[m] = 0u; mn[m] = PG_NEVER; }
         if (c.n <= PG_FILL_SMALL) {   // a warp per instance
             const u32 inst = lt * 8u + (threadIdx.x >> 5), lane = threadIdx.x & 31u;
             if (inst >= c.n_inst) continue;
-            const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
-            u32 cnt = 0, mn = PG_NEVER;
-            for (u32 i = lane; i < c.n; i += 32u) {
-                if (rs[so + i] != rt[to + i]) { cnt++; mn = min(mn, i); }
-            }
-            cnt = __reduce_add_sync(0xffffffffu, cnt);
-            mn = __reduce_min_sync(0xffffffffu, mn);
-            if (lane == 0 && cnt) {
-                atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step].count, (u64)cnt);
-                atomicMin(&mm_key[c.mm0 + (u64)inst * c.mm_step], ((u64)c.gid << 32) | mn);
+            PgCmpRows w;
+            pg_cmp_rows(c, R, inst, w);
+            for (u32 i = lane; i < c.n; i += 32u) pg_cmp_cell(w, i, cnt, mn);
+#pragma unroll
+            for (u32 a = 0; a + 1 < PG_MAXK; a++) {
+                if (a + 1 >= c.nm) break;
+                const u32 t = __reduce_add_sync(0xffffffffu, cnt[a]);
+                const u32 x = __reduce_min_sync(0xffffffffu, mn[a]);
+                if (lane == 0 && t) {
+                    atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step + (u64)c.kid[a] * PG_NK].count, (u64)t);
+                    atomicMin(&mm_key[c.mm0 + (u64)inst * c.mm_step + c.kid[a]], ((u64)c.gid << 32) | x);
+                }
             }
             continue;
         }
         const u32 nch = (c.n + PG_FILL_CHUNK - 1u) / PG_FILL_CHUNK;
         const u32 inst = lt / nch, w0 = (lt - inst * nch) * PG_FILL_CHUNK, w1 = min(c.n, w0 + PG_FILL_CHUNK);
-        if (threadIdx.x == 0) { s_cnt = 0; s_min = PG_NEVER; }
+        if (threadIdx.x < PG_MAXK) { s_cnt[threadIdx.x] = 0; s_min[threadIdx.x] = PG_NEVER; }
         __syncthreads();
-        const u64 so = c.src_off + (u64)inst * c.src_stride, to = c.tgt_off + (u64)inst * c.tgt_stride;
-        u32 cnt = 0, mn = PG_NEVER;
-        for (u32 i = w0 + threadIdx.x; i < w1; i += blockDim.x) {
-            if (rs[so + i] != rt[to + i]) { cnt++; mn = min(mn, i); }
+        PgCmpRows w;
+        pg_cmp_rows(c, R, inst, w);
+        for (u32 i = w0 + threadIdx.x; i < w1; i += blockDim.x) pg_cmp_cell(w, i, cnt, mn);
+#pragma unroll
+        for (u32 a = 0; a + 1 < PG_MAXK; a++) {
+            if (a + 1 >= c.nm) break;
+            const u32 t = __reduce_add_sync(0xffffffffu, cnt[a]);
+            const u32 x = __reduce_min_sync(0xffffffffu, mn[a]);
+            if ((threadIdx.x & 31) == 0 && t) { atomicAdd(&s_cnt[a], t); atomicMin(&s_min[a], x); }
         }
-        cnt = __reduce_add_sync(0xffffffffu, cnt);
-        mn = __reduce_min_sync(0xffffffffu, mn);
-        if ((threadIdx.x & 31) == 0 && cnt) { atomicAdd(&s_cnt, cnt); atomicMin(&s_min, mn); }
         __syncthreads();
-        if (threadIdx.x == 0 && s_cnt) {
-            atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step].count, (u64)s_cnt);
-            atomicMin(&mm_key[c.mm0 + (u64)inst * c.mm_step], ((u64)c.gid << 32) | s_min);
+        if (threadIdx.x + 1 < c.nm && s_cnt[threadIdx.x]) {
+            const u32 a = threadIdx.x;
+            atomicAdd(&slots[c.slot0 + (u64)inst * c.slot_step + (u64)c.kid[a] * PG_NK].count, (u64)s_cnt[a]);
+            atomicMin(&mm_key[c.mm0 + (u64)inst * c.mm_step + c.kid[a]], ((u64)c.gid << 32) | s_min[a]);
         }
         __syncthreads();
     }
 }
 
-__device__ __forceinline__ u32 pg_cmp_lw(const PgRegions& R, u32 r, u32 has, u64 lw, u64 inst, u64 stride, u32 addr) {
-    return has ? R.r[r][lw + inst * stride + addr] - 1u : PG_NEVER;
+__device__ __forceinline__ u32 pg_cmp_val(const PgCmp& c, const PgRegions& R, u32 m, u32 inst, u32 i) {
+    return R.r[c.region[m]][c.off[m] + (u64)inst * c.stride[m] + i];
 }
+__device__ __forceinline__ u32 pg_cmp_lw(const PgCmp& c, const PgRegions& R, u32 m, u32 inst, u32 i) {
+    return ((c.lw_flags >> m) & 1u) ? R.r[c.region[m]][c.lw[m] + (u64)inst * c.stride[m] + i] - 1u : PG_NEVER;
+}
+__device__ __forceinline__ u32 pg_cmp_site(const PgCmp& c, u32 b) { return c.nmode ? c.kid[b] : PG_NEVER; }
 
-// K3b: among the pairs (i, j) that mismatch at kernel i's minimum cell, the minimum
-// (tid_b, site) - the remaining fields of the X16 minimum event.
+// K3b: for each member a whose kernel's minimum mismatching cell lies in this job's array,
+// the minimum (tid_b, site) over the pairs (a, b) that differ there - the remaining fields
+// of the X16 minimum event.
 __global__ void __launch_bounds__(128) pg_compare_pick(const PgCmp* __restrict__ jobs, const PgRegions R,
                                                        const u64* mm_key, u64* mm2) {
-    const PgCmp c = jobs[blockIdx.y];
+    const PgCmp& c = jobs[blockIdx.y];
     const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
     if (inst >= c.n_inst) return;
-    const u64 mi = c.mm0 + (u64)inst * c.mm_step;
-    const u64 k = mm_key[mi];
-    if (k == ~0ull || (u32)(k >> 32) != c.gid) return;
-    const u32 addr = (u32)k;
-    if (addr >= c.n) return;
-    const u32 a = R.r[c.src_r][c.src_off + (u64)inst * c.src_stride + addr];
-    const u32 b = R.r[c.tgt_r][c.tgt_off + (u64)inst * c.tgt_stride + addr];
-    if (a == b) return;
-    const u32 tb = pg_cmp_lw(R, c.tgt_r, c.lw_flags & 2u, c.tgt_lw, inst, c.tgt_stride, addr);
-    atomicMin(&mm2[mi], ((u64)tb << 32) | c.site);
+    for (u32 a = 0; a + 1 < c.nm; a++) {
+        const u64 mi = c.mm0 + (u64)inst * c.mm_step + c.kid[a];
+        const u64 k = mm_key[mi];
+        if (k == ~0ull || (u32)(k >> 32) != c.gid) continue;
+        const u32 i = (u32)k;
+        if (i >= c.size[a]) continue;
+        const u32 va = pg_cmp_val(c, R, a, inst, i);
+        for (u32 b = a + 1; b < c.nm; b++) {
+            if (!pg_pair(c, a, b, i) || pg_cmp_val(c, R, b, inst, i) == va) continue;
+            atomicMin(&mm2[mi], ((u64)pg_cmp_lw(c, R, b, inst, i) << 32) | pg_cmp_site(c, b));
+        }
+    }
 }
 
-// K3c: fill the MISMATCH record of every failing (instance, kernel i) from the pair the
-// pick chose.
+// K3c: fill each failing (instance, kernel kid[a]) MISMATCH record from the pair the pick chose.
 __global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__ jobs, const PgRegions R,
                                                        PgSlot* slots, const u64* mm_key, const u64* mm2) {
-    const PgCmp c = jobs[blockIdx.y];
+    const PgCmp& c = jobs[blockIdx.y];
     const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
     if (inst >= c.n_inst) return;
-    const u64 mi = c.mm0 + (u64)inst * c.mm_step;
-    const u64 k = mm_key[mi];
-    if (k == ~0ull || (u32)(k >> 32) != c.gid) return;
-    const u32 addr = (u32)k;
-    if (addr >= c.n) return;
-    const u32 a = R.r[c.src_r][c.src_off + (u64)inst * c.src_stride + addr];
-    const u32 b = R.r[c.tgt_r][c.tgt_off + (u64)inst * c.tgt_stride + addr];
-    const u32 tb = pg_cmp_lw(R, c.tgt_r, c.lw_flags & 2u, c.tgt_lw, inst, c.tgt_stride, addr);
-    if (a == b || mm2[mi] != (((u64)tb << 32) | c.site)) return;
-    PgSlot* s = &slots[c.slot0 + (u64)inst * c.slot_step];
-    s->f[0] = 0xFFFFu;
-    s->f[1] = c.gid;
-    s->f[2] = addr;
-    s->f[3] = pg_cmp_lw(R, c.src_r, c.lw_flags & 1u, c.src_lw, inst, c.src_stride, addr);
-    s->f[4] = tb;
-    s->f[5] = c.site;
-    s->f[6] = a;
-    s->f[7] = b;
-    s->has = 1u;
+    for (u32 a = 0; a + 1 < c.nm; a++) {
+        const u64 mi = c.mm0 + (u64)inst * c.mm_step + c.kid[a];
+        const u64 k = mm_key[mi];
+        if (k == ~0ull || (u32)(k >> 32) != c.gid) continue;
+        const u32 i = (u32)k;
+        if (i >= c.size[a]) continue;
+        const u32 va = pg_cmp_val(c, R, a, inst, i);
+        for (u32 b = a + 1; b < c.nm; b++) {
+            if (!pg_pair(c, a, b, i)) continue;
+            const u32 vb = pg_cmp_val(c, R, b, inst, i);
+            const u32 tb = pg_cmp_lw(c, R, b, inst, i);
+            if (vb == va || mm2[mi] != (((u64)tb << 32) | pg_cmp_site(c, b))) continue;
+            PgSlot* s = &slots[c.slot0 + (u64)inst * c.slot_step + (u64)c.kid[a] * PG_NK];
+            s->f[0] = 0xFFFFu;
+            s->f[1] = c.gid;
+            s->f[2] = i;
+            s->f[3] = pg_cmp_lw(c, R, a, inst, i);
+            s->f[4] = tb;
+            s->f[5] = pg_cmp_site(c, b);
+            s->f[6] = va;
+            s->f[7] = vb;
+            s->has = 1u;
+            break;
+        }
+    }
 }
 
 // K2b: flag every instance in which some global cell written by the kernel was

@@ -172,18 +172,27 @@ struct PgLock {
     u32 n_inst, nblocks, size, rounds, arr_slot, pad;
 };
 
-// K3 (pg_compare) job: one compared global array of one pair of kernels (i, j) for n_inst
-// consecutive instances of one launch (H7).
+// K3 (pg_compare) job: one global array (pair-level id) of one launch segment, compared
+// between every pair of the kernels that have it (H7): member m is kernel kid[m]'s copy.  A
+// pair (a, b), a < b, is compared when pair_mask has bit a * PG_MAXK + b (one of the two
+// declares it out / inout), on the cells below both declared sizes; its mismatches are
+// events of kernel kid[a]'s MISMATCH slot.  Each cell is read once per member, not once per
+// pair.
 struct PgCmp {
-    u64 src_off, tgt_off;        // u32-word offsets of instance 0 in their regions
-    u64 src_stride, tgt_stride;  // per-instance strides of the regions the offsets point into
-    u64 src_lw, tgt_lw;          // last-writer words of instance 0 (arena regions only)
-    u64 slot0, slot_step;        // MISMATCH slot of (instance 0, kernel i) and stride
-    u32 inst0, n_inst, gid, n;
-    u32 src_r, tgt_r;            // regions: arena of kernel i / j, or PG_R_INPUT (array only read)
+    u64 off[PG_MAXK];            // value words of instance 0 in the member's region
+    u64 stride[PG_MAXK];         // per-instance stride of that region
+    u64 lw[PG_MAXK];             // last-writer words of instance 0 (members with bit m of lw_flags)
+    u32 region[PG_MAXK];         // arena of kernel k, or PG_R_INPUT (array only read)
+    u32 size[PG_MAXK];           // the member's declared size
+    u32 kid[PG_MAXK];            // the member's kernel index (record slot)
+    u64 pair_mask;
+    u64 slot0, slot_step;        // MISMATCH slot of (instance 0, kernel 0) and the instance stride
+    u64 mm0, mm_step;            // min-cell words of (instance 0, kernel 0) and the instance stride
+    u32 inst0, n_inst, gid, n;   // n: cells scanned (the largest member size)
+    u32 nm;                      // members
+    u32 lw_flags;
+    u32 nmode;                   // N-kernel check: record site = the other kernel; else PG_NEVER
     u32 task0;                   // first CTA task (pg_fill_tasks(n, n_inst))
-    u32 site;                    // record site field: j in N-kernel checks, PG_NEVER for a pair
-    u64 mm0, mm_step;            // per-(instance, kernel i) minimum-cell words of instance 0, stride
-    u32 lw_flags;                // bit 0 / 1: the source / target side has last-writer words (else NONE)
-    u32 pad;
+    u32 pad_writes_;             // (planner scratch: members that declare the array out / inout)
+    u32 pad_;
 };
