@@ -95,6 +95,11 @@ typedef struct {
     int64_t *d_counts;                         /* borrowed device int64[16]: [0] instances (X19), [1+k] events of kind k,
                                                   [11] records, [12] failing (launch, seed) instances,
                                                   [13] IR operations executed (PG_CHK_OPCOUNT only) */
+    uint32_t key_launch0, key_seed0;           /* added to the launch index and the seed index of every key and
+                                                  record: a sub-space (some launches x a seed range, e.g. one item
+                                                  of a greedy (launch, seed) assignment, §8(e)) reports the keys of
+                                                  the whole space, so sub-space results merge like rank shards.
+                                                  0 for a whole space */
 } pg_space;
 
 /* One counterexample record (X16): the minimum event of its (launch, seed,

@@ -934,6 +934,7 @@ enum { IN_RAND32 = 0, IN_BITS01 = 1, IN_RANGE = 2 };
 enum { MODE_EQUIV = 0, MODE_RACES = 1, MODE_BANKS = 2 };
 static const uint32_t NONE32 = 0xFFFFFFFFu;
 static const uint32_t ROUND_END = 0xFFFFu;     /* round field of MISMATCH / XB records */
+static const uint32_t ROUND_LIMIT = 0xFFFEu;   /* rounds 0..0xFFFD run; threads still live then stop (LIMIT) */
 
 /* One record per slot (instance, kernel, kind): the minimum event by
  * (round, array, addr, tid_a, tid_b, site, val_a, val_b) plus the event count
@@ -1682,7 +1683,14 @@ struct Exec {
                 for (uint32_t i = 0; i < T; i++) any |= !th[i].exited;
                 cur_round++;
                 if (!any) break;
-                if (cur_round >= 0xFFFFu) throw Error(E_LIMIT, "more than 65534 rounds in a block");
+                if (cur_round >= ROUND_LIMIT) {   /* X19: the round field saturates (X16 keys keep 16 bits) */
+                    for (uint32_t i = 0; i < T; i++)
+                        if (!th[i].exited) {
+                            event(K_LIMIT, ROUND_LIMIT, NONE32, 0, b * T + i, NONE32, NONE32, 3, 0);
+                            th[i].exited = true;
+                        }
+                    break;
+                }
             }
             res.instances += (uint64_t)T * cur_round;   /* X19: threads x rounds per block */
         }

@@ -192,8 +192,8 @@ struct PgCold {     // per-emulated-thread state that lives in local memory
                                  // degree, ...), so one word per kind (local-memory footprint) ...
     u32 vbx;                     // ... unless two events with equal fields 0..5 but different val_b
     u32 ebvs[PG_NK][PG_MS];      //     met (bit k): then val_b per seed here
-    u64 epk[PG_NK];              // pg_pack of ebest[kind] (one 64-bit compare decides most events)
 #endif
+    u64 epk[PG_NK];              // pg_pack of ebest[kind] (one 64-bit compare decides most events)
 };
 
 __device__ __forceinline__ bool pg_lex_less(const u32* a, const u32* b) {
@@ -225,11 +225,20 @@ __device__ __forceinline__ u64 pg_pack(const u32* f) {
 }
 // Records an event of `kind`; `evm` is the caller's event mask (PgT::evm).  Returns the
 // kind's bit, which the caller ORs into its mask.
+// The packed prefix pg_pack of the kind's minimum (epk) decides most comparisons with one
+// 64-bit load: a thread's events mostly arrive in increasing order (round first).
 __device__ __noinline__ u32 pg_event(PgCold& c, u32 evm, u32 kind, u32 round, u32 arr, u32 addr, u32 ta, u32 tb,
                                      u32 site, u32 va, u32 vb) {
     u32 e[8] = {round, arr, addr, ta, tb, site, va, vb};
     const u32 has = (evm >> kind) & 1u;
-    if (!has || pg_lex_less(e, c.ebest[kind])) {
+    const u64 pk = pg_pack(e);
+    bool take = !has;
+    if (has) {
+        const u64 bp = c.epk[kind];
+        take = pk < bp || (pk == bp && pg_lex_less(e, c.ebest[kind]));
+    }
+    if (take) {
+        c.epk[kind] = pk;
 #pragma unroll
         for (int i = 0; i < 8; i++) c.ebest[kind][i] = e[i];
     }
@@ -1345,6 +1354,16 @@ __device__ __noinline__ void pg_snapshot(const PgC& C, const PgT& t) {
 }
 #endif
 
+// X19: a block runs rounds 0..0xFFFD; threads still live at round 0xFFFE (the round field
+// of X16 keys has 16 bits, 0xFFFF marks MISMATCH / XB) stop with a LIMIT event (val_a 3).
+#define PG_ROUND_LIMIT 0xFFFEu
+__device__ __forceinline__ void pg_round_limit(const PgC& C, PgT& t, PgCold& c) {
+    if (C.round >= PG_ROUND_LIMIT && t.live) {
+        PG_EVENT(t, c, PGK_LIMIT, PG_ROUND_LIMIT, PG_NEVER, 0u, t.gtid, PG_NEVER, PG_NEVER, 3u, 0u);
+        t.live = 0u;
+    }
+}
+
 // End of a round when the rounds of a block run inline (K::run, one emulated thread
 // per lane): barrier, claims, barrier, checks, then the early-exit vote.  Unless LAST,
 // begin the next round and return whether any thread of the CTA is still live.
@@ -1356,6 +1375,7 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
     // once some thread flagged a race the item stops (every instance of the warp / CTA is
     // re-run exactly, so finishing it would be wasted work)
     C.round++;
+    pg_round_limit(C, t, c);
     if (warp_blocks) __syncwarp();
     if (LAST) {
         if (!warp_blocks) __syncthreads();
@@ -1396,6 +1416,7 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
     pg_snapshot(C, t);
 #endif
     C.round++;
+    pg_round_limit(C, t, c);
     if (LAST) return false;
     const int more = warp_blocks ? __any_sync(PG_FULL, t.live) : __syncthreads_or((int)t.live);
     if (!more) return false;
@@ -1871,10 +1892,12 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
                 t.bid[0] = blk & (pg_sL.gdim[0] - 1u);
                 t.bid[1] = (blk >> gsh0) & (pg_sL.gdim[1] - 1u);
                 t.bid[2] = blk >> (gsh0 + gsh1);
-            } else {
-                t.bid[0] = blk % pg_sL.gdim[0];
-                t.bid[1] = (blk / pg_sL.gdim[0]) % pg_sL.gdim[1];
-                t.bid[2] = blk / (pg_sL.gdim[0] * pg_sL.gdim[1]);
+            } else {   // (blk < 2^20: division by multiply-high with the launch's magic numbers)
+                const u32 q0 = (u32)(((u64)blk * pg_sL.gmag0) >> 40);
+                const u32 q01 = (u32)(((u64)blk * pg_sL.gmag01) >> 40);
+                t.bid[0] = blk - q0 * pg_sL.gdim[0];
+                t.bid[1] = q0 - q01 * pg_sL.gdim[1];
+                t.bid[2] = q01;
             }
             t.live = inst_ok && t.tlin < T_ && blk_ok;
             t.gtid = blk * T_ + t.tlin;
@@ -1949,6 +1972,9 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
             }
 #endif
             C.round++;
+#pragma unroll
+            for (u32 v = 0; v < PG_VMAX; v++)
+                if (v < V) pg_round_limit(C, T[v], Cd[v]);
 #if PG_FAST
             u32 fl = 0;
 #pragma unroll

@@ -414,12 +414,12 @@ __device__ __forceinline__ bool kind_failing(u32 kind, u32 banks_mode) {
 // K4a: per instance (launch, local seed m): count non-empty slots, fold counts
 // and keys into the summary (X16/X17).
 __global__ void __launch_bounds__(256) pg_summarize(const PgSlot* __restrict__ slots, u32 n_inst, u32 n_local,
-                                                    u32 rank, u32 world, u32 banks_mode, u32 nks, u32* inst_nrec,
-                                                    long long* first_key, long long* counts) {
+                                                    u32 rank, u32 world, u32 banks_mode, u32 nks, u32 l0, u32 s0,
+                                                    u32* inst_nrec, long long* first_key, long long* counts) {
     const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
     if (inst >= n_inst) return;
-    const u32 li = inst / n_local, m = inst % n_local;
-    const u32 sj = rank + m * world;
+    const u32 li = l0 + inst / n_local, m = inst % n_local;
+    const u32 sj = s0 + rank + m * world;
     u32 n = 0, failing = 0;
     for (u32 k = 0; k < nks; k++) {
         for (u32 kind = 0; kind < PG_NK; kind++) {
@@ -484,13 +484,13 @@ struct PgCexDev {
 // The run's record count (its own records, before any cross-rank reduction of the counters)
 // goes to *total.
 __global__ void __launch_bounds__(256) pg_compact(const PgSlot* __restrict__ slots, u32 n_inst, u32 n_local,
-                                                  u32 rank, u32 world, u32 nks, const u32* inst_nrec,
+                                                  u32 rank, u32 world, u32 nks, u32 l0, u32 s0, const u32* inst_nrec,
                                                   const u64* offsets, PgCexDev* out, u64 cap, u64* total) {
     const u32 inst = blockIdx.x * blockDim.x + threadIdx.x;
     if (inst == 0) *total = offsets[n_inst - 1] + inst_nrec[n_inst - 1];
     if (inst >= n_inst) return;
-    const u32 li = inst / n_local, m = inst % n_local;
-    const u32 sj = rank + m * world;
+    const u32 li = l0 + inst / n_local, m = inst % n_local;
+    const u32 sj = s0 + rank + m * world;
     u64 o = offsets[inst];
     for (u32 k = 0; k < nks; k++) {
         for (u32 kind = 0; kind < PG_NK; kind++) {
@@ -692,20 +692,20 @@ cudaError_t reset_counters(long long* first_key, long long* counts, cudaStream_t
 }
 
 cudaError_t summarize_scan(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, u32 banks_mode,
-                           u32 nks, u32* inst_nrec, u64* offsets, long long* first_key, long long* counts,
-                           cudaStream_t st) {
+                           u32 nks, u32 l0, u32 s0, u32* inst_nrec, u64* offsets, long long* first_key,
+                           long long* counts, cudaStream_t st) {
     if (!n_inst) return cudaSuccess;
-    pg_summarize<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, banks_mode, nks,
+    pg_summarize<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, banks_mode, nks, l0, s0,
                                                        inst_nrec, first_key, counts);
     pg_scan<<<1, 1024, 0, st>>>(inst_nrec, offsets, n_inst);
     return cudaGetLastError();
 }
 
-cudaError_t compact(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, u32 nks,
+cudaError_t compact(const PgSlot* slots, u32 n_inst, u32 n_local, u32 rank, u32 world, u32 nks, u32 l0, u32 s0,
                     const u32* inst_nrec, const u64* offsets, void* out, u64 cap, u64* total, cudaStream_t st) {
     if (!n_inst) return cudaSuccess;
-    pg_compact<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, nks, inst_nrec, offsets,
-                                                     (PgCexDev*)out, cap, total);
+    pg_compact<<<(n_inst + 255) / 256, 256, 0, st>>>(slots, n_inst, n_local, rank, world, nks, l0, s0, inst_nrec,
+                                                     offsets, (PgCexDev*)out, cap, total);
     return cudaGetLastError();
 }
 

@@ -61,6 +61,8 @@ struct PgLaunchK {
     u64 off_step0;                           // data-flow mode: per-block first round step (arena words), ~0 absent
     u64 off_hist, off_hround;                // VC-literal mode: [block][round < 64][thread][1 + W_max] logged
                                              // writes, [block] rounds (arena words), ~0 absent
+    u64 gmag0, gmag01;                       // ceil(2^40 / d) for d = gdim.x and gdim.x * gdim.y: block index ->
+                                             // bid by multiply and shift (exact for block indices < 2^20)
     PgArr arr[PG_MAXARR];
 };
 

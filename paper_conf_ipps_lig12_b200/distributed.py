@@ -39,3 +39,39 @@ def first_witness(first_key: int):
         return None
     return {"launch": first_key >> 45, "seed_idx": (first_key >> 24) & 0x1FFFFF, "kernel": (first_key >> 20) & 0xF,
             "kind": (first_key >> 16) & 0xF, "round": first_key & 0xFFFF}
+
+
+def greedy_assignment(costs: Sequence[float], n_seeds: Sequence[int], world: int, chunk: int = 0):
+    """where seeds are few per launch (C4's exhaustive 0/1 sets, one-seed
+    runs), round-robin seed shards leave ranks idle; instead the (launch, seed) instances
+    are assigned greedily by cost (longest processing time first: items sorted by cost, each
+    to the least-loaded rank).  costs[l] = cost of one (launch l, seed) instance (e.g.
+    threads x rounds x ops), n_seeds[l] = its seeds.  Items are (launch, seed range) chunks
+    of `chunk` seeds (default: enough to give every rank several items).  Returns, per rank,
+    a list of (launch, seed0, seed1) in launch order - each becomes a sub-space whose
+    pg_space.key_launch0 / key_seed0 put its records at their global keys."""
+    if world < 1:
+        raise ValueError("world >= 1")
+    total = sum(int(s) for s in n_seeds)
+    chunk = chunk or max(1, total // (8 * world))
+    items = []
+    for l, (c, ns) in enumerate(zip(costs, n_seeds)):
+        for a in range(0, int(ns), chunk):
+            b = min(int(ns), a + chunk)
+            items.append((float(c) * (b - a), l, a, b))
+    items.sort(key=lambda x: (-x[0], x[1], x[2]))
+    load = [0.0] * world
+    out = [[] for _ in range(world)]
+    for c, l, a, b in items:
+        r = min(range(world), key=lambda i: (load[i], i))
+        load[r] += c
+        out[r].append((l, a, b))
+    for r in range(world):   # merge adjacent seed ranges of a launch, launch order
+        merged = []
+        for l, a, b in sorted(out[r]):
+            if merged and merged[-1][0] == l and merged[-1][2] == a:
+                merged[-1] = (l, merged[-1][1], b)
+            else:
+                merged.append((l, a, b))
+        out[r] = merged
+    return out

@@ -37,7 +37,8 @@ class PgSpace(ctypes.Structure):
                 ("input_mode", ctypes.c_uint32), ("input_range", ctypes.c_uint32), ("bits", ctypes.c_uint32),
                 ("checks", ctypes.c_uint32), ("bank_model", ctypes.c_uint32), ("max_cex", ctypes.c_uint32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("cuda_stream", ctypes.c_void_p),
-                ("d_first_key", ctypes.c_void_p), ("d_counts", ctypes.c_void_p)]
+                ("d_first_key", ctypes.c_void_p), ("d_counts", ctypes.c_void_p),
+                ("key_launch0", ctypes.c_uint32), ("key_seed0", ctypes.c_uint32)]
 
 
 LOCK_FIELDS = ("launch", "seed_idx", "block", "round", "array", "addr", "val_src", "val_tgt", "written_src",
@@ -231,6 +232,8 @@ class Space:
     stream: int = 0                 # cudaStream_t as an integer (torch.cuda.Stream.cuda_stream)
     first_key: object = None        # torch int64[11] on the device (optional)
     counts: object = None           # torch int64[16] on the device (optional)
+    key_launch0: int = 0            # launch / seed index offsets of the keys (a sub-space of a larger space)
+    key_seed0: int = 0
 
     def marshal(self):
         # (the launch arrays are built once per Space object: a Space re-used for every step
@@ -257,6 +260,7 @@ class Space:
         sp.cuda_stream = self.stream or None
         sp.d_first_key = _counter_ptr(self.first_key, 11, "first_key")
         sp.d_counts = _counter_ptr(self.counts, 16, "counts")
+        sp.key_launch0, sp.key_seed0 = self.key_launch0, self.key_seed0
         return sp, (ls, lt)
 
 

@@ -80,3 +80,27 @@ def test_oracle_check_parallel_equals_serial(oracle, W):
     a = oracle.check(*args, n_seeds=5, checks=w.checks, cap=1 << 20)
     b = oracle.check_parallel(*args, n_seeds=5, checks=w.checks, cap=1 << 20, processes=3)
     assert a["records"] == b["records"] and a["counts"] == b["counts"] and a["first_key"] == b["first_key"]
+
+
+def test_greedy_assignment_covers_and_balances():
+    from paper_conf_ipps_lig12_b200 import distributed as D
+    # C4's exhaustive 0/1 sets: n = 2, 4, 8, 16 threads with 2^n seeds, cost ~ n log^2 n
+    ns = [2, 4, 8, 16]
+    costs = [n * max(1, (n.bit_length() - 1)) ** 2 for n in ns]
+    seeds = [1 << n for n in ns]
+    for world in (1, 2, 3, 8):
+        asg = D.greedy_assignment(costs, seeds, world)
+        seen = {}
+        for r, items in enumerate(asg):
+            for l, a, b in items:
+                for s in range(a, b):
+                    assert (l, s) not in seen
+                    seen[(l, s)] = r
+        assert len(seen) == sum(seeds)                       # every (launch, seed) exactly once
+        loads = [sum(costs[l] * (b - a) for l, a, b in items) for items in asg]
+        chunk = max(1, sum(seeds) // (8 * world))
+        biggest = max(costs) * chunk
+        assert max(loads) - min(loads) <= biggest           # LPT: within one item of each other
+    # round-robin over seeds would leave ranks 4..7 idle on the 4-seed launch; greedy spreads it
+    asg = D.greedy_assignment([1.0], [4], 8, chunk=1)
+    assert sum(1 for items in asg if items) == 4

@@ -94,3 +94,19 @@ def test_repeated_and_interleaved_checks(env, oracle, W):  # noqa: F811
     first = [pgvc.check_equiv(s, t, sp).collect() for sp in (a, b)]
     again = [pgvc.check_equiv(s, t, sp).collect() for sp in (b, a, b)]
     assert again[1] == first[0] and again[0] == first[1] and again[2] == first[1]
+
+
+@pytest.mark.parametrize("T", [2, 48, 512])
+def test_round_limit(env, oracle, T):  # noqa: F811
+    # X19 round limit: 70000 barrier rounds; every live thread stops at round 0xFFFE with a
+    # LIMIT record, as in the oracle (the optimistic pass flags, the exact re-run records)
+    k = """
+    kernel spin_sync(global out int o[n], unsigned n) {
+      for (unsigned i = 0; i < 70000; i++) { sync; }
+      o[bid.x * bdim.x + tid.x] = 1;
+    }
+    """
+    ls = [((2, 1, 1), (T, 1, 1), (2 * T,))]
+    ref, recs, summ, _ = run_pair(env, oracle, k, None, ls, mode=1, n_seeds=2)
+    assert_same(ref, recs, summ)
+    assert summ["per_kind"][9] == 2 * 2 * T

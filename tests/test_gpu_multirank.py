@@ -97,3 +97,41 @@ def test_bench_world2_branch_matches_world1(env):  # noqa: F811
     # 2 ranks x 4 seeds (seeds r, r+2, ...) = the 1-rank run's 8 seeds: same H9-reduced summary
     assert two["check"] == one["check"]
     assert two["value"] > 0 and two["e2e"]["value"] > 0
+
+
+@pytest.mark.timeout(900)
+def test_greedy_assignment_subspaces_merge_like_the_whole(env, oracle, W):  # noqa: F811
+    """§8(e) greedy (launch, seed) split of C4's exhaustive 0/1 sets (n = 2, 4, 8: 4, 16, 256
+    seeds): each rank runs its items as sub-spaces whose key_launch0 / key_seed0 give the
+    records their global keys; merged over 3 ranks (MIN keys, SUM counts, records in key
+    order) they equal one run per launch - and the oracle's records with the same offsets."""
+    pgvc, torch = env
+    from paper_conf_ipps_lig12_b200 import distributed as D
+    ws = W.c4("bits", max_log_n=3)
+    src, tgt = pgvc.load_ir(W.subject(ws[0].src)), pgvc.load_ir(W.subject(ws[0].tgt))
+    st = torch.cuda.current_stream().cuda_stream
+    costs = [l.bdim[0] * (l.bdim[0].bit_length() ** 2) for w in ws for l in w.launch_src]
+    seeds = [w.n_seeds for w in ws]
+
+    def run(l, a, b):
+        w = ws[l]
+        sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=b - a, seed_base=a, input_mode=1, checks=w.checks,
+                        stream=st, key_launch0=l, key_seed0=a)
+        recs, summ = pgvc.check_equiv(src, tgt, sp).collect(cap=1 << 20)
+        return recs, summ
+
+    whole = [run(l, 0, seeds[l]) for l in range(len(ws))]
+    want_recs = sorted((r for recs, _ in whole for r in recs), key=lambda r: r[0])
+    want_inst = sum(s["instances"] for _, s in whole)
+    want_first = min(s["first_key"] for _, s in whole)
+    asg = D.greedy_assignment(costs, seeds, 3, chunk=8)
+    got = [run(l, a, b) for items in asg for l, a, b in items]
+    assert sorted((r for recs, _ in got for r in recs), key=lambda r: r[0]) == want_recs
+    assert sum(s["instances"] for _, s in got) == want_inst
+    assert min(s["first_key"] for _, s in got) == want_first
+    # the oracle on the same sub-spaces, its keys offset by hand (it has no key offsets)
+    for l, w in enumerate(ws):
+        ref = oracle.check(W.subject(w.src), W.subject(w.tgt), w.launch_src, w.launch_tgt, n_seeds=seeds[l],
+                           input_mode=1, checks=w.checks, cap=1 << 20)
+        mine = [r for r in want_recs if r[3] == l]
+        assert [(r[0] + (l << 45),) + tuple(r[1:3]) + (r[3] + l,) + tuple(r[4:]) for r in ref["records"]] == mine

@@ -1,7 +1,8 @@
 """Multi-seed lanes: the optimistic pass of a seed-oblivious kernel
-carries 4 seeds per lane.  Seed counts that are not multiples of 4 leave ragged seed
-groups; races, OOB and uninitialised reads inside a group flag all its instances for the
-exact single-seed re-run.  Every case must equal the oracle bit for bit."""
+carries PG_MS = 8 seeds per lane (PGVC_MS).  Seed counts that are not multiples of 8 leave
+ragged seed groups; races, OOB and uninitialised reads inside a group flag all its
+instances for the exact re-run, which runs the same seed groups (multi-seed exact
+protocol).  Every case must equal the oracle bit for bit."""
 import pytest
 
 from test_gpu_parity import assert_same, env, run_pair  # noqa: F401  (fixture re-export)

@@ -257,3 +257,19 @@ def test_loop_fuel_limit_record(oracle):
     _, fin, counts = oracle.exec_kernel(k, one(bdim=(3, 1, 1)), 0)
     assert int(fin[0][0]) == 1                       # thread 0 finished; 1 and 2 never reached the store
     assert counts[0] == 3
+
+
+def test_round_limit_record(oracle):
+    # X19 / X16: keys keep 16 round bits (0xFFFF marks MISMATCH / XB), so a block runs rounds
+    # 0..0xFFFD; threads still live when round 0xFFFE would begin stop with a LIMIT event
+    # (round 0xFFFE, their gtid, val_a = 3).  Instances: T x 0xFFFE rounds.
+    k = """
+    kernel spin_sync(global out int o[4]) { for (unsigned i = 0; i < 70000; i++) { sync; } o[tid.x] = 1; }
+    """
+    r = oracle.check(k, None, [one(bdim=(2, 1, 1), gdim=(2, 1, 1))], mode=oracle.MODE_RACES,
+                     checks=oracle.RACE | oracle.OOB)
+    (rec,) = r["records"]
+    d = dict(zip(oracle.REC_FIELDS, rec))
+    assert (d["kind"], d["round"], d["array"], d["addr"], d["tid_a"], d["tid_b"], d["site"], d["val_a"], d["count"]) == \
+        (9, 0xFFFE, 0xFFFFFFFF, 0, 0, 0xFFFFFFFF, 0xFFFFFFFF, 3, 4)
+    assert r["counts"][0] == 4 * 0xFFFE
