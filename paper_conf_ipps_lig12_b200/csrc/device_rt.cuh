@@ -271,6 +271,18 @@ __device__ __forceinline__ u32 pg_owner_step(u32 own) { return 0xFFFFFu - (own >
 
 __device__ __forceinline__ u32* pg_sh(const PgT& t, u32 off) { return (u32*)(pg_dsmem + t.sg + off); }
 
+// Optimistic pass, reader side of the RW check (one atomic per read): a cell of the round's
+// parity set keeps the LAST reader's stamp (R, atomicExch; the rmin words) and a flag that
+// a second, different reader of the same round came by (M = the round's smax tag; the rmax
+// words).  After the barrier the writer w sees a race iff R is of this round and
+// (R != w or M flagged): with two or more distinct readers some exchange returns another
+// reader's stamp of the round and sets M; a single reader r != w leaves R = r.
+__device__ __forceinline__ void pg_fread(u32* R, u32* M, u32 smax, u32 tlin) {
+    const u32 me = smax | tlin;
+    const u32 old = atomicExch(R, me);
+    if (old != me && (old ^ me) < 0x1000u) *M = smax;
+}
+
 #ifndef PG_FAST
 #define PG_FAST 0
 #endif
@@ -507,8 +519,7 @@ __device__ __forceinline__ u32 pg_ld_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
     if (pe & inb) {
         if (RD && PG_T > 1u) {
             const u32 so = C.par * PG_SH(A, size) + flat;
-            atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + so, C.smin | t.tlin);
-            atomicMax(pg_sh(t, PG_SH(A, s_rmax)) + so, C.smax | t.tlin);
+            pg_fread(pg_sh(t, PG_SH(A, s_rmin)) + so, pg_sh(t, PG_SH(A, s_rmax)) + so, C.smax, t.tlin);
         }
         own = pg_sh(t, PG_SH(A, s_own))[flat];
         v = pg_sh(t, PG_SH(A, s_val))[flat];
@@ -600,12 +611,11 @@ __device__ __forceinline__ void pg_commit_sh(const PgC& C, PgT& t, PgCold& c, u3
     pg_sh(t, PG_SH(A, s_val))[flat] = val;
     pg_fcount(t);
 }
-// after the round's barrier: readers of a cell this thread wrote in round `step`
-// readers of the round other than this thread: the max reader stamp is of this round and
-// the min / max reader stamps are not both this thread's
-__device__ __forceinline__ u32 pg_fast_rw(const PgC& C, const PgT& t, u32 rmin, u32 rmax) {
-    const u32 a = rmax ^ (C.smax | t.tlin);
-    return (a < 0x1000u) & ((a | (rmin ^ (C.smin | t.tlin))) != 0u);
+// after the round's barrier: a reader of the round other than this thread (pg_fread: the
+// last reader word R is of this round and another thread's, or a second reader was flagged)
+__device__ __forceinline__ u32 pg_fast_rw(const PgC& C, const PgT& t, u32 R, u32 M) {
+    const u32 a = R ^ (C.smax | t.tlin);
+    return (a < 0x1000u) & ((a != 0u) | (M == C.smax));
 }
 template <int A>
 __device__ __forceinline__ void pg_fcheck_sh(const PgC& C, PgT& t, u32 flat) {
@@ -699,8 +709,7 @@ __device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     if (pe & inb) {
         if (RD && PG_T > 1u) {
             const u32 so = C.par * PG_SH(A, size) + flat;
-            atomicMin(pg_sh(t, PG_SH(A, s_rmin)) + so, C.smin | t.tlin);
-            atomicMax(pg_sh(t, PG_SH(A, s_rmax)) + so, C.smax | t.tlin);
+            pg_fread(pg_sh(t, PG_SH(A, s_rmin)) + so, pg_sh(t, PG_SH(A, s_rmax)) + so, C.smax, t.tlin);
         }
         own = pg_sh(t, PG_SH(A, s_own))[flat];
         pg_vld(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
@@ -752,8 +761,7 @@ __device__ __forceinline__ void pg_ld_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     pg_xb_mark_ms<A>(t, flat);
     if (RD && PG_T > 1u) {
         const u64 so = (u64)C.par * PG_ARR(A).size + flat;
-        atomicMin(t.arena + PG_ARR(A).off_rmin + so, C.smin | t.tlin);
-        atomicMax(t.arena + PG_ARR(A).off_rmax + so, C.smax | t.tlin);
+        pg_fread(t.arena + PG_ARR(A).off_rmin + so, t.arena + PG_ARR(A).off_rmax + so, C.smax, t.tlin);
     }
     const u64 st = pg_sL.arena_stride;
     PG_S_LOOP if (_s < t.nsv) v[_s] = t.arena[_s * st + PG_ARR(A).off_val + flat];
@@ -777,12 +785,10 @@ __device__ __forceinline__ void pg_st_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
         *own = me;
     }
     const u64 st = pg_sL.arena_stride;
-    PG_S_LOOP {
-        if (_s < t.nsv) {
-            t.arena[_s * st + PG_ARR(A).off_val + flat] = val[_s];
-            t.arena[_s * st + PG_ARR(A).off_lw + flat] = t.gtid + 1u;
-        }
-    }
+    PG_S_LOOP if (_s < t.nsv) t.arena[_s * st + PG_ARR(A).off_val + flat] = val[_s];
+    // the last writer is the same in every seed of the group (same accesses): the group's first
+    // arena keeps it (K2b and K3 read it there)
+    t.arena[PG_ARR(A).off_lw + flat] = t.gtid + 1u;
     pg_fcount(t);
 }
 template <int A>
@@ -1113,8 +1119,7 @@ __device__ __forceinline__ u32 pg_ld_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
 #if PG_FAST
     if (RD && PG_T > 1u) {
         const u64 so = (u64)C.par * PG_ARR(A).size + flat;
-        atomicMin(t.arena + PG_ARR(A).off_rmin + so, C.smin | t.tlin);
-        atomicMax(t.arena + PG_ARR(A).off_rmax + so, C.smax | t.tlin);
+        pg_fread(t.arena + PG_ARR(A).off_rmin + so, t.arena + PG_ARR(A).off_rmax + so, C.smax, t.tlin);
     }
     return t.arena[PG_ARR(A).off_val + flat];
 #else

@@ -194,7 +194,8 @@ __device__ __forceinline__ u32 pg_cmp_val(const PgCmp& c, const PgRegions& R, u3
     return R.r[c.region[m]][c.off[m] + (u64)inst * c.stride[m] + i];
 }
 __device__ __forceinline__ u32 pg_cmp_lw(const PgCmp& c, const PgRegions& R, u32 m, u32 inst, u32 i) {
-    return ((c.lw_flags >> m) & 1u) ? R.r[c.region[m]][c.lw[m] + (u64)inst * c.stride[m] + i] - 1u : PG_NEVER;
+    const u32 ig = c.lwg[m] > 1u ? inst - inst % c.lwg[m] : inst;
+    return ((c.lw_flags >> m) & 1u) ? R.r[c.region[m]][c.lw[m] + (u64)ig * c.stride[m] + i] - 1u : PG_NEVER;
 }
 __device__ __forceinline__ u32 pg_cmp_site(const PgCmp& c, u32 b) { return c.nmode ? c.kid[b] : PG_NEVER; }
 

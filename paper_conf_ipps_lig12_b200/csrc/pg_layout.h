@@ -187,6 +187,8 @@ struct PgCmp {
     u32 region[PG_MAXK];         // arena of kernel k, or PG_R_INPUT (array only read)
     u32 size[PG_MAXK];           // the member's declared size
     u32 kid[PG_MAXK];            // the member's kernel index (record slot)
+    u32 lwg[PG_MAXK];            // multi-seed group of the member's launch: its last-writer words live
+                                 // in the group's first instance (the same cells in every seed)
     u64 pair_mask;
     u64 slot0, slot_step;        // MISMATCH slot of (instance 0, kernel 0) and the instance stride
     u64 mm0, mm_step;            // min-cell words of (instance 0, kernel 0) and the instance stride
