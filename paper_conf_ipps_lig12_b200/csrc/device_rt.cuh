@@ -87,7 +87,8 @@ __device__ __forceinline__ u32 pg_not(u32 a) { return pg_m(~a); }
 
 // ------------------------------------------------------------------ state
 extern __shared__ __align__(16) unsigned char pg_dsmem[];  // group regions | site stats | group counters
-__shared__ PgLaunchK pg_sL;                                 // this CTA's launch descriptor
+__shared__ __align__(16) PgLaunchK pg_sL;                   // this CTA's launch descriptor (TMA bulk copy)
+__shared__ __align__(8) u64 pg_sBar;                        // its mbarrier (complete_tx of the bulk copy)
 __shared__ PgWork pg_sW;                                    // this CTA's work item
 
 #define PG_ARR(A) (pg_sL.arr[A])
@@ -1730,8 +1731,28 @@ __device__ __forceinline__ void pg_barrier_div(const PgC& C, PgT* T, PgCold* Cd,
 }
 #endif
 
+// The launch descriptor (the IR's layout constants: array offsets, sizes, strides, 2.3 KB)
+// of the item is staged into shared memory by the TMA engine: one thread arms the CTA's
+// mbarrier with the byte count and issues a 1-D cp.async.bulk; every thread waits on the
+// barrier's phase (one phase per item).
+__device__ __forceinline__ u32 pg_smem_addr(const void* p) { return (u32)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void pg_desc_bulk_issue(const PgLaunchK* src) {
+    const u32 bar = pg_smem_addr(&pg_sBar), dst = pg_smem_addr(&pg_sL), bytes = (u32)sizeof(PgLaunchK);
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // (earlier generic reads of pg_sL)
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void pg_desc_bulk_wait(u32 phase) {
+    const u32 bar = pg_smem_addr(&pg_sBar);
+    u32 done = 0;
+    while (!done)
+        asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                     : "=r"(done) : "r"(bar), "r"(phase) : "memory");
+}
+
 template <class K>
-__device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
+__device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi, u32& phase) {
     __shared__ u32 s_flag;
     if (P.seq) {
         // re-runs: only items with a flagged instance (seq 1: a global cell shared between
@@ -1746,12 +1767,12 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi) {
         if (!s_flag) return;
     }
     {
-        const u32* src = (const u32*)&P.launches[P.work[wi].launch];
-        u32* dst = (u32*)&pg_sL;
-        for (u32 i = threadIdx.x; i < sizeof(PgLaunchK) / 4; i += blockDim.x) dst[i] = src[i];
+        if (threadIdx.x == 0) pg_desc_bulk_issue(&P.launches[P.work[wi].launch]);
         const u32* ws = (const u32*)&P.work[wi];
         u32* wd = (u32*)&pg_sW;
         for (u32 i = threadIdx.x; i < sizeof(PgWork) / 4; i += blockDim.x) wd[i] = ws[i];
+        pg_desc_bulk_wait(phase);
+        phase ^= 1u;
     }
 #if PG_DATAFLOW
     if (threadIdx.x == 0) pg_sDf = PgDf{P.df_rows, P.df_count, P.seed_base, P.df_cap};
@@ -2162,8 +2183,14 @@ __device__ __forceinline__ void pg_main(const PgParams& P) {
     if (P.seq && P.flag_any && *(volatile const u32*)P.flag_any == 0u) return;   // nothing to re-run
     const bool listed = P.work_count != nullptr;
     const u32 n = listed ? *P.work_count : P.n_work ? P.n_work : blockIdx.x + 1u;
+    if (threadIdx.x == 0) {   // the descriptor's mbarrier: one arrival (the issuing thread) per phase
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(pg_smem_addr(&pg_sBar)) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    u32 phase = 0;
     for (u32 i = blockIdx.x; i < n; i += gridDim.x) {   // (one call site: one inlined copy)
-        pg_item<K>(P, listed ? P.work_list[i] : i);
+        pg_item<K>(P, listed ? P.work_list[i] : i, phase);
         __syncthreads();
     }
 }
