@@ -523,10 +523,16 @@ __global__ void __launch_bounds__(256) pg_compact(const PgSlot* __restrict__ slo
 // Before the exact re-run of flagged instances: clear their record slots (this kernel)
 // and their instance counts.
 __global__ void __launch_bounds__(256) pg_reset_flagged(const u32* flags, u32 n_inst, const u64* inst_slot0,
-                                                        u32 kernel, PgSlot* slots, u64* inst_cnt) {
+                                                        u32 kernel, PgSlot* slots, u64* inst_cnt,
+                                                        u32* flag_count) {
     const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
     if (!flags[n_inst]) return;   // (the batch's any-flagged word)
-    if (i >= n_inst || !flags[i]) return;
+    const u32 f = i < n_inst && flags[i] != 0u;
+    if (flag_count) {   // flagged instances of the check (the planner's choice of main pass)
+        const u32 c = __popc(__ballot_sync(0xffffffffu, f));
+        if ((threadIdx.x & 31u) == 0u && c) atomicAdd(flag_count, c);
+    }
+    if (!f) return;
     inst_cnt[i] = 0ull;
     PgSlot* s = slots + inst_slot0[i] + (u64)kernel * PG_NK;
     for (u32 k = 0; k < PG_NK; k++) {
@@ -619,9 +625,10 @@ cudaError_t gen_inputs(const PgFill* jobs, u32 n_jobs, u32 task_base, u32 n_task
 }
 
 cudaError_t reset_flagged(const u32* flags, u32 n_inst, const u64* inst_slot0, u32 kernel, PgSlot* slots,
-                          u64* inst_cnt, cudaStream_t st) {
+                          u64* inst_cnt, u32* flag_count, cudaStream_t st) {
     if (!n_inst) return cudaSuccess;
-    pg_reset_flagged<<<(n_inst + 255) / 256, 256, 0, st>>>(flags, n_inst, inst_slot0, kernel, slots, inst_cnt);
+    pg_reset_flagged<<<(n_inst + 255) / 256, 256, 0, st>>>(flags, n_inst, inst_slot0, kernel, slots, inst_cnt,
+                                                           flag_count);
     return cudaGetLastError();
 }
 
