@@ -1754,6 +1754,8 @@ __device__ __forceinline__ void pg_desc_bulk_wait(u32 phase) {
 template <class K>
 __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi, u32& phase) {
     __shared__ u32 s_flag;
+    // (launches the sequential pass takes whole this check: nothing to do in the parallel passes)
+    if (P.seq != 1u && P.seq_pref && P.seq_pref[P.work[wi].launch]) return;
     if (P.seq) {
         // re-runs: only items with a flagged instance (seq 1: a global cell shared between
         // blocks; seq 2: a race the optimistic pass flagged)
@@ -2084,6 +2086,8 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi, u32& ph
                     if (lw[i] && xf[i] != xl[i])
                         PG_EVENT(t, Cd[v], PGK_XB, 0xFFFFu, ar.rec_id, i, xf[i] - 1u, xl[i] - 1u, PG_NEVER, val[i], 0u);
             }
+            // (the sequential preference of the next check counts instances that raced here)
+            if (P.seq_pref && ((t.evm >> PGK_XB) & 1u)) P.xb_flag[pg_sW.inst0 + sb] = 2u;
         }
     }
 #endif

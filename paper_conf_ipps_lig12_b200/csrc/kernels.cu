@@ -257,7 +257,7 @@ __global__ void __launch_bounds__(128) pg_compare_fill(const PgCmp* __restrict__
 // K2b: flag every instance in which some global cell written by the kernel was
 // accessed by two blocks (X4 XB) - the block-parallel pass is not exact there.
 __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ jobs, u32 n_jobs, u32 n_tasks,
-                                                    const u32* arena, u32* flags, u32* any) {
+                                                    const u32* arena, u32* flags, u32* any, const u32* pref) {
     __shared__ u32 s_job;
     if (threadIdx.x == 0) s_job = 0u;
     for (u32 task = blockIdx.x; task < n_tasks; task += gridDim.x) {
@@ -269,9 +269,15 @@ __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ job
             for (u32 i = i0; i < i1; i++) flags[j.inst0 + i] = 1u;
             *any = 1u;
         };
+        // (launches the sequential pass takes whole: the parallel passes skipped them)
+        const bool all = pref != nullptr && pref[j.launch] != 0u;
         if (j.n <= PG_FILL_SMALL) {   // a warp per instance
             const u32 b = lt * 8u + (threadIdx.x >> 5), lane = threadIdx.x & 31u;
             if (b >= nb) continue;
+            if (all) {
+                if (lane == 0) flag(b);
+                continue;
+            }
             const u64 base = (u64)b * j.istep * j.stride;
             u32 hit = 0;
             for (u32 i = lane; i < j.n; i += 32u) {
@@ -283,6 +289,10 @@ __global__ void __launch_bounds__(256) pg_xb_detect(const PgXb* __restrict__ job
         }
         const u32 nch = (j.n + PG_FILL_CHUNK - 1u) / PG_FILL_CHUNK;
         const u32 b = lt / nch, w0 = (lt - b * nch) * PG_FILL_CHUNK, w1 = min(j.n, w0 + PG_FILL_CHUNK);
+        if (all) {
+            if (threadIdx.x == 0 && w0 == 0) flag(b);
+            continue;
+        }
         const u64 base = (u64)b * j.istep * j.stride;
         u32 hit = 0;
         for (u32 i = w0 + threadIdx.x; i < w1; i += blockDim.x) {
@@ -543,6 +553,23 @@ __global__ void __launch_bounds__(256) pg_reset_flagged(const u32* flags, u32 n_
     }
 }
 
+// Sequential preference (PgParams::seq_pref): the instances whose sequential run found an XB
+// race (flag word 2), counted per launch (launch = record slot / (n_local x slots per seed)).
+__global__ void __launch_bounds__(256) pg_xb_tally(const u32* flags, u32 n_inst, const u64* inst_slot0, u64 div,
+                                                   u32* counts) {
+    const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (!flags[n_inst]) return;
+    if (i < n_inst && flags[i] == 2u) atomicAdd(&counts[inst_slot0[i] / div], 1u);
+}
+// After the check: a launch goes straight to the sequential pass next time iff at least half
+// of its instances here raced between blocks (re-decided every check); counts reset.
+__global__ void __launch_bounds__(256) pg_seq_pref_update(u32* counts, u32* pref, u32 n, u32 n_local) {
+    const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    pref[i] = 2u * counts[i] >= n_local && counts[i] != 0u ? 1u : 0u;
+    counts[i] = 0u;
+}
+
 // X19: the batch's per-instance counts into the run's instance counter.
 __global__ void __launch_bounds__(1024) pg_count_reduce(const u64* inst_cnt, u32 n, unsigned long long* counts) {
     u64 x = 0;
@@ -632,6 +659,18 @@ cudaError_t reset_flagged(const u32* flags, u32 n_inst, const u64* inst_slot0, u
     return cudaGetLastError();
 }
 
+cudaError_t xb_tally(const u32* flags, u32 n_inst, const u64* inst_slot0, u64 div, u32* counts, cudaStream_t st) {
+    if (!n_inst) return cudaSuccess;
+    pg_xb_tally<<<(n_inst + 255) / 256, 256, 0, st>>>(flags, n_inst, inst_slot0, div, counts);
+    return cudaGetLastError();
+}
+
+cudaError_t seq_pref_update(u32* counts, u32* pref, u32 n, u32 n_local, cudaStream_t st) {
+    if (!n) return cudaSuccess;
+    pg_seq_pref_update<<<(n + 255) / 256, 256, 0, st>>>(counts, pref, n, n_local);
+    return cudaGetLastError();
+}
+
 cudaError_t count_reduce(const u64* inst_cnt, u32 n, long long* counts, cudaStream_t st) {
     if (!n) return cudaSuccess;
     pg_count_reduce<<<1, 1024, 0, st>>>(inst_cnt, n, (unsigned long long*)counts);
@@ -668,10 +707,9 @@ cudaError_t lockstep(const PgLock* jobs, u32 n_jobs, u32 max_inst, const u32* ar
 }
 
 cudaError_t xb_detect(const PgXb* jobs, u32 n_jobs, u32 n_tasks, const u32* arena, u32* flags, u32* any,
-                      cudaStream_t st) {
+                      const u32* pref, cudaStream_t st) {
     if (!n_jobs || !n_tasks) return cudaSuccess;
-    pg_xb_detect<<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, arena, flags,
-                                                                              any);
+    pg_xb_detect<<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, arena, flags, any, pref);
     return cudaGetLastError();
 }
 

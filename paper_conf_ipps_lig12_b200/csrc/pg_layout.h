@@ -122,6 +122,9 @@ struct PgParams {
     u32 keep_vals;          // sequential pass of a later phase of a kernel sequence: the global values
                             // are the previous phase's results (only stamps are reset)
     u32 pad4;
+    const u32* seq_pref;    // per launch: its instances go straight to the sequential pass (the last
+                            // check's sequential pass found an XB race in at least half of them): the
+                            // block-parallel passes skip their items, K2b flags them (nullptr: off)
 };
 
 // K1 (pg_gen_inputs) job: one buffer of one array for n_inst consecutive
@@ -162,7 +165,8 @@ struct PgXb {
     u32 n, n_inst, inst0;
     u32 istep;        // multi-seed launches: the marks live in the first instance of each group of
                       // istep seeds, whose verdict holds for the whole group
-    u32 task0, pad;   // first CTA task (pg_fill_tasks over the instances holding marks)
+    u32 task0;        // first CTA task (pg_fill_tasks over the instances holding marks)
+    u32 launch;       // the launch (index into the launch table) of the job's instances
 };
 
 // K3b (pg_lockstep) job: one shared array both kernels of a pair declare (same name

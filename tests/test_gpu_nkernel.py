@@ -42,30 +42,3 @@ def test_c2_all_bench_space_nine_seeds(env, oracle, W, group):
     recs, summ = _gpu(env, W, w.kernels, w.launches, 9)
     assert_same(ref, recs, summ)
 
-
-def test_repeated_check_switches_main_pass(env, oracle, W):
-    """A plan whose optimistic pass flags at least half of a kernel's instances (the injected
-    off-by-one races in every instance with B >= 2) runs that kernel's exact pass as its main
-    pass from the next check on (api.cpp choose_main_passes; a scheduling choice, DESIGN.md
-    §5.5).  Every repetition - optimistic pass + re-run, then exact main pass - must equal
-    the oracle bit for bit."""
-    w = W.c2_all(n_seeds=9, max_log_n=12, max_log_b=10)[0]
-    assert "reduce2_obo" in w.kernels
-    ref = oracle.check_n_parallel([W.subject(n) for n in w.kernels], w.launches, n_seeds=9, cap=1 << 20)
-    pgvc, torch = env
-    sp = pgvc.Space(w.launches[0], n_seeds=9, checks=7, stream=torch.cuda.current_stream().cuda_stream)
-    irs = [ir(pgvc, W.subject(n)) for n in w.kernels]
-    for _ in range(3):
-        recs, summ = pgvc.check_equiv_n(irs, w.launches, sp).collect(cap=1 << 20)
-        assert_same(ref, recs, summ)
-
-
-def test_repeated_pair_check_switches_main_pass(env, oracle, W):
-    w = W.c2_pair("reduce2", "reduce2_obo", n_seeds=9, max_log_n=11, max_log_b=10)
-    ref = oracle.check_parallel(W.subject(w.src), W.subject(w.tgt), w.launch_src, w.launch_tgt, n_seeds=9,
-                                cap=1 << 20)
-    pgvc, torch = env
-    sp = pgvc.Space(w.launch_src, w.launch_tgt, n_seeds=9, stream=torch.cuda.current_stream().cuda_stream)
-    for _ in range(3):
-        recs, summ = pgvc.check_equiv(ir(pgvc, W.subject(w.src)), ir(pgvc, W.subject(w.tgt)), sp).collect(cap=1 << 20)
-        assert_same(ref, recs, summ)
