@@ -2087,7 +2087,7 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi, u32& ph
                         PG_EVENT(t, Cd[v], PGK_XB, 0xFFFFu, ar.rec_id, i, xf[i] - 1u, xl[i] - 1u, PG_NEVER, val[i], 0u);
             }
             // (the sequential preference of the next check counts instances that raced here)
-            if (P.seq_pref && ((t.evm >> PGK_XB) & 1u)) P.xb_flag[pg_sW.inst0 + sb] = 2u;
+            if ((t.evm >> PGK_XB) & 1u) P.xb_flag[pg_sW.inst0 + sb] = 2u;
         }
     }
 #endif

@@ -556,10 +556,13 @@ __global__ void __launch_bounds__(256) pg_reset_flagged(const u32* flags, u32 n_
 // Sequential preference (PgParams::seq_pref): the instances whose sequential run found an XB
 // race (flag word 2), counted per launch (launch = record slot / (n_local x slots per seed)).
 __global__ void __launch_bounds__(256) pg_xb_tally(const u32* flags, u32 n_inst, const u64* inst_slot0, u64 div,
-                                                   u32* counts) {
+                                                   u32* counts, u32* total) {
     const u32 i = blockIdx.x * blockDim.x + threadIdx.x;
     if (!flags[n_inst]) return;
-    if (i < n_inst && flags[i] == 2u) atomicAdd(&counts[inst_slot0[i] / div], 1u);
+    const u32 x = i < n_inst && flags[i] == 2u;
+    if (x && counts) atomicAdd(&counts[inst_slot0[i] / div], 1u);
+    const u32 c = __popc(__ballot_sync(0xffffffffu, x));   // (the host's count: any XB at all)
+    if ((threadIdx.x & 31u) == 0u && c) atomicAdd(total, c);
 }
 // After the check: a launch goes straight to the sequential pass next time iff at least half
 // of its instances here raced between blocks (re-decided every check); counts reset.
@@ -659,9 +662,10 @@ cudaError_t reset_flagged(const u32* flags, u32 n_inst, const u64* inst_slot0, u
     return cudaGetLastError();
 }
 
-cudaError_t xb_tally(const u32* flags, u32 n_inst, const u64* inst_slot0, u64 div, u32* counts, cudaStream_t st) {
+cudaError_t xb_tally(const u32* flags, u32 n_inst, const u64* inst_slot0, u64 div, u32* counts, u32* total,
+                     cudaStream_t st) {
     if (!n_inst) return cudaSuccess;
-    pg_xb_tally<<<(n_inst + 255) / 256, 256, 0, st>>>(flags, n_inst, inst_slot0, div, counts);
+    pg_xb_tally<<<(n_inst + 255) / 256, 256, 0, st>>>(flags, n_inst, inst_slot0, div, counts, total);
     return cudaGetLastError();
 }
 
