@@ -484,7 +484,8 @@ def main():
                   "n_fail": int(cnts[-1][12].item()), "records": int(cnts[-1][11].item()),
                   "per_kind": [int(x) for x in cnts[-1][1:11].tolist()]},
     }
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and WL in ("c2", "c2n"):
+        # (the oracle sample is C2's: the other configs are parity cases, not the headline)
         # like for like: the oracle and the GPU on the same bounded sample (C2 with N <= 2^k, seeds
         # 0..S-1), then the oracle's number as the CPU baseline
         inst, dt, cores, sample = oracle_sample(max_log_n=args.ref_log_n, n_seeds=args.ref_seeds)

@@ -4,9 +4,10 @@
 #   2. DRAM bytes and time of every evaluation-kernel launch (roofline "traffic")
 #   3. one `--set full` capture of the top evaluation-kernel launch (source-level, -lineinfo)
 set -u
-# ncu cannot profile the kernel nodes of a graph that has conditional nodes: profile with the
-# re-run blocks as plain (early-exiting) launches instead
-export PGVC_COND=0
+# ncu cannot profile the kernel nodes of a graph that has conditional nodes: profile the checks
+# eagerly, the host deciding each conditional block from its flag word - the same launches the
+# graphs run
+export PGVC_GRAPH=0 PGVC_COND=host
 OUT=${1:-gpurun_out/prof}
 WL=${2:-c2}
 mkdir -p "$OUT/src"
