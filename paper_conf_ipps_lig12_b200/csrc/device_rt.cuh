@@ -36,6 +36,14 @@
 #ifndef PG_DIVBAR
 #define PG_DIVBAR 0    // a barrier under thread-dependent control: per-thread resume points (X18)
 #endif
+#ifndef PG_VCLIT
+#define PG_VCLIT 0
+#endif
+// the exact protocol claims a cell when the store enters the write log (the claim words are
+// separate from the committed-owner words loads consult), so a round needs two barriers, not
+// three; the diagnostic variants (data-flow dump, VC-literal, lock-step) and run-time barrier
+// divergence keep the separate claim phase
+#define PG_CAS (!PG_FAST && !PG_DATAFLOW && !PG_VCLIT && !PG_DIVBAR && !PG_LOCKSTEP)
 #define PG_MSX (PG_MS > 1 && !PG_FAST)
 #define PG_S_LOOP _Pragma("unroll") for (u32 _s = 0; _s < (u32)PG_MS; _s++)
 
@@ -398,21 +406,48 @@ __device__ __noinline__ u32 pg_log_write_slow(u32 nlog, PgCold& c, u32 cell, u32
     return nlog + 1u;
 }
 
-__device__ __forceinline__ void pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell, u32 val, u32 site, u32 rec,
-                                             u32 flat) {
+// Returns 1 when the cell entered the log (its first store of the round: the claim).
+__device__ __forceinline__ u32 pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell, u32 val, u32 site, u32 rec,
+                                            u32 flat) {
     if (t.nlog == 0u) {
         t.l0cell = cell;
         t.l0val = val;
         t.l0site = site;
         t.nlog = 1u;
+        return 1u;
     } else if (t.l0cell == cell) {
         t.l0val = val;
         t.l0site = site;
     } else {
         const u32 n = pg_log_write_slow(t.nlog, c, cell, val, site);
         if (n == PG_NEVER) PG_EVENT(t, c, PGK_LIMIT, C.round, rec, flat, t.gtid, PG_NEVER, site, 1, 0);
-        else t.nlog = n;
+        else {
+            const u32 fresh = n != t.nlog;
+            t.nlog = n;
+            return fresh;
+        }
     }
+    return 0u;
+}
+
+// Claim (exact protocol): atomicMin on the cell's claim stamp (newest round wins over stale
+// stamps, the min tid wins within the round) plus atomicMax for WW detection.  Shared arrays
+// claim into s_clm when claims happen at store time (PG_CAS: s_own keeps the committed owner
+// that loads of the round consult), into s_own otherwise; global owner words are not read
+// during a round outside the data-flow dump.
+template <int A>
+__device__ __forceinline__ void pg_claim_sh(const PgC& C, const PgT& t, u32 flat) {
+    atomicMin(pg_sh(t, PG_CAS ? PG_SH(A, s_clm) : PG_SH(A, s_own)) + flat, pg_stamp_min(C, t));
+#if PG_RACECHK
+    if (PG_T > 1u) atomicMax(pg_sh(t, PG_SH(A, s_wmax)) + flat, pg_stamp_max(C, t));
+#endif
+}
+template <int A>
+__device__ __forceinline__ void pg_claim_gt(const PgC& C, const PgT& t, u32 flat) {
+    atomicMin(t.arena + PG_ARR(A).off_own + flat, pg_stamp_min(C, t));
+#if PG_RACECHK
+    if (PG_T > 1u) atomicMax(t.arena + PG_ARR(A).off_wmax + flat, pg_stamp_max(C, t));
+#endif
 }
 
 #if PG_DATAFLOW
@@ -423,9 +458,6 @@ struct PgDf {
     u32 cap;
 };
 __shared__ PgDf pg_sDf;  // data-flow recorder of this CTA
-#ifndef PG_VCLIT
-#define PG_VCLIT 0
-#endif
 #define PG_HIST_R 64u   // rounds per block the VC-literal history keeps
 #if PG_VCLIT
 // GPU VC-literal mode: the
@@ -654,7 +686,8 @@ __device__ __forceinline__ void pg_st_sh(PgC& C, PgT& t, PgCold& c, u64* ss, u32
 #if PG_FAST
     pg_commit_sh<A, RDA>(C, t, c, flat, val);
 #else
-    pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+    if (pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat) && PG_CAS && PG_T > 1u)
+        pg_claim_sh<A>(C, t, flat);
 #endif
 }
 
@@ -872,21 +905,27 @@ __device__ __noinline__ u32 pg_log_write_slow_ms(u32 nlog, PgCold& c, u32 cell, 
     c.lsite[nlog] = (u16)site;
     return nlog + 1u;
 }
-__device__ __forceinline__ void pg_log_write_ms(PgC& C, PgT& t, PgCold& c, u32 cell, const u32 (&val)[PG_MS],
-                                                u32 site, u32 rec, u32 flat) {
+__device__ __forceinline__ u32 pg_log_write_ms(PgC& C, PgT& t, PgCold& c, u32 cell, const u32 (&val)[PG_MS],
+                                               u32 site, u32 rec, u32 flat) {
     if (t.nlog == 0u) {
         t.l0cell = cell;
         PG_S_LOOP t.l0v[_s] = val[_s];
         t.l0site = site;
         t.nlog = 1u;
+        return 1u;
     } else if (t.l0cell == cell) {
         PG_S_LOOP t.l0v[_s] = val[_s];
         t.l0site = site;
     } else {
         const u32 n = pg_log_write_slow_ms(t.nlog, c, cell, val, site);
         if (n == PG_NEVER) PG_EVENT(t, c, PGK_LIMIT, C.round, rec, flat, t.gtid, PG_NEVER, site, 1, 0);
-        else t.nlog = n;
+        else {
+            const u32 fresh = n != t.nlog;
+            t.nlog = n;
+            return fresh;
+        }
     }
+    return 0u;
 }
 template <int A, bool RD, bool LOG>
 __device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
@@ -936,7 +975,8 @@ __device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 #endif
         return;
     }
-    pg_log_write_ms(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+    if (pg_log_write_ms(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat) && PG_CAS && PG_T > 1u)
+        pg_claim_sh<A>(C, t, flat);
 }
 template <int A>
 __device__ __forceinline__ void pg_xb_mark_ms(const PgT& t, u32 flat) {
@@ -988,7 +1028,8 @@ __device__ __forceinline__ void pg_st_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
         return;
     }
     pg_xb_mark_ms<A>(t, flat);
-    pg_log_write_ms(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+    if (pg_log_write_ms(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat) && PG_CAS && PG_T > 1u)
+        pg_claim_gt<A>(C, t, flat);
 }
 template <int A>
 __device__ __forceinline__ void pg_ld_gi_ms(PgC& C, PgT& t, PgCold& c, u64* ss, u32 pe, u32 flat, u32 site,
@@ -1039,8 +1080,11 @@ __device__ __forceinline__ void pg_check_sh_ms(const PgC& C, PgT& t, PgCold& c, 
         pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
         return;
     }
-    const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
-    if (own == pg_stamp_min(C, t)) pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
+    const u32 own = pg_sh(t, PG_CAS ? PG_SH(A, s_clm) : PG_SH(A, s_own))[flat];
+    if (own == pg_stamp_min(C, t)) {
+        pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
+        if (PG_CAS) pg_sh(t, PG_SH(A, s_own))[flat] = own;
+    }
 #if PG_RACECHK
     if (PG_T > 1u) {
         const u32 wmax = pg_sh(t, PG_SH(A, s_wmax))[flat];
@@ -1175,7 +1219,8 @@ __device__ __forceinline__ void pg_st_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32
         pg_fcount(t);
     }
 #else
-    pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat);
+    if (pg_log_write(C, t, c, ((u32)A << 24) | flat, val, site, PG_ARR(A).rec_id, flat) && PG_CAS && PG_T > 1u)
+        pg_claim_gt<A>(C, t, flat);
 #endif
 }
 
@@ -1224,20 +1269,6 @@ __device__ __forceinline__ void pg_tick(PgC& C, PgT& t, PgCold& c, u32 act) {
 // min tid wins within the round).  Check (after a barrier): the owner commits
 // its value (and, for global arrays, itself as last writer); with race checks
 // the owner reports WW, and the thread the X16 rule names tid_a reports RW.
-template <int A>
-__device__ __forceinline__ void pg_claim_sh(const PgC& C, const PgT& t, u32 flat) {
-    atomicMin(pg_sh(t, PG_SH(A, s_own)) + flat, pg_stamp_min(C, t));
-#if PG_RACECHK
-    if (PG_T > 1u) atomicMax(pg_sh(t, PG_SH(A, s_wmax)) + flat, pg_stamp_max(C, t));
-#endif
-}
-template <int A>
-__device__ __forceinline__ void pg_claim_gt(const PgC& C, const PgT& t, u32 flat) {
-    atomicMin(t.arena + PG_ARR(A).off_own + flat, pg_stamp_min(C, t));
-#if PG_RACECHK
-    if (PG_T > 1u) atomicMax(t.arena + PG_ARR(A).off_wmax + flat, pg_stamp_max(C, t));
-#endif
-}
 
 __device__ __noinline__ u32 pg_race_check(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 evm, u32 val,
                                           u32 site, u32 rec, u32 flat, u32 own, u32 wmax, u32 has_readers, u32 rmin,
@@ -1265,8 +1296,11 @@ __device__ __forceinline__ void pg_check_sh(const PgC& C, PgT& t, PgCold& c, u32
         pg_sh(t, PG_SH(A, s_val))[flat] = val;
         return;
     }
-    const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
-    if (own == pg_stamp_min(C, t)) pg_sh(t, PG_SH(A, s_val))[flat] = val;
+    const u32 own = pg_sh(t, PG_CAS ? PG_SH(A, s_clm) : PG_SH(A, s_own))[flat];
+    if (own == pg_stamp_min(C, t)) {
+        pg_sh(t, PG_SH(A, s_val))[flat] = val;
+        if (PG_CAS) pg_sh(t, PG_SH(A, s_own))[flat] = own;
+    }
 #if PG_RACECHK
     if (PG_T > 1u) {
         const u32 wmax = pg_sh(t, PG_SH(A, s_wmax))[flat];
@@ -1324,7 +1358,7 @@ template <class K>
 __device__ __forceinline__ void pg_claim_all(const PgC& C, const PgT& t, const PgCold& c) {
     // a 1-thread block is the only writer of its cells in the round (other blocks sharing a
     // global cell are an XB race and re-run sequentially): the check commits directly
-    if (t.nlog == 0u || PG_T == 1u) return;
+    if (t.nlog == 0u || PG_T == 1u || PG_CAS) return;   // (PG_CAS: claimed at store time)
     K::claim_one(C, t, t.l0cell);
     for (u32 i = 1; i < t.nlog; i++) K::claim_one(C, t, c.lcell[i]);
 }
@@ -1411,8 +1445,10 @@ __device__ __forceinline__ bool pg_round_end(PgC& C, PgT& t, PgCold& c, u32& ali
     return true;
 #else
     if (warp_blocks) __syncwarp(); else __syncthreads();
+#if !PG_CAS
     pg_claim_all<K>(C, t, c);
     if (warp_blocks) __syncwarp(); else __syncthreads();
+#endif
     pg_check_all<K>(C, t, c);
 #if PG_VCLIT
     pg_hist_put(C, t, c);
@@ -1986,12 +2022,14 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi, u32& ph
             }
 #else
             if (warp_blocks) __syncwarp(); else __syncthreads();
+#if !PG_CAS
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;
                 pg_claim_all<K>(C, T[v], Cd[v]);
             }
             if (warp_blocks) __syncwarp(); else __syncthreads();
+#endif
 #pragma unroll
             for (u32 v = 0; v < PG_VMAX; v++) {
                 if (v >= V) break;

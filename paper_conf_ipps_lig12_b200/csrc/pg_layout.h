@@ -37,6 +37,8 @@ struct PgArr {
     u32 flags;      // bit0: reader stamps present (array read and written, race checks on)
     // shared arrays: byte offsets in the group's shared region
     u32 s_val, s_own, s_wmax, s_rmin, s_rmax;
+    u32 s_clm;      // claims of the round (exact protocol with claims at store time; s_own then
+                    // holds the committed owner only, which loads of the same round consult)
     u32 rsets;      // reader-stamp sets (rmin/rmax hold rsets x size words): 2 when the optimistic
                     // pass checks a round's readers after the next barrier (set = step & 1)
     // global arrays written by the kernel: u32-word offsets in the instance arena

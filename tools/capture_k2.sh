@@ -3,7 +3,7 @@
 # bench step (indices count pgk_eval launches only, as in k2_metrics.csv).
 #   tools/capture_k2.sh OUT WORKLOAD IDX [IDX ...]
 set -u
-export PGVC_COND=0   # (ncu cannot profile kernel nodes of graphs with conditional nodes)
+export PGVC_GRAPH=0 PGVC_COND=host   # (the launches the conditional nodes run, as plain launches ncu can profile)
 OUT=$1; WL=$2; shift 2
 mkdir -p "$OUT/src"
 for IDX in "$@"; do
