@@ -65,6 +65,13 @@ WORKLOADS = {
 }
 WL = "c2n"
 
+# SURVEY.md §8(d) "Algorithmic work per instance": IR integer ops per (thread, round) counted
+# from the paper's code - the per-unit figure the roofline's `achieved` is built on (reduction
+# round ~10; transposes 13 / 14; scan round 13-17; bitonic round 10-11; matmul: naive
+# 10 ops/k x K + 10 in 1 round, tiled 2 x 14 + 2 x 10 ops/k x 32 + 10 over 5 rounds, K = 64)
+SURVEY_OPS = {"c2": 10.0, "c2n": 10.0, "c1": 13.5, "c5t": 13.5, "c3": 15.0, "c4": 10.5,
+              "c5m": (10 * 64 + 10 + 2 * 14 + 2 * 10 * 32 + 10) / 6.0}
+
 
 def workload_desc():
     return WORKLOADS[WL][0] % SEEDS_PER_GPU
@@ -450,11 +457,15 @@ def main():
     value = inst_total / (dev_ms / 1000.0)
     e2e = inst_total / wall_s
     sm_max = clk.get("sm_max_mhz") or measured_peaks().get("sm_max_mhz", 1965.0)
-    # roofline (per GPU): useful IR integer ops of this rank's step / K2 busy time, against
-    # the measured integer peak of both pipes (alu: IADD3/LOP3/SHF/ISETP, fma: IMAD)
+    # roofline (per GPU): algorithmic work of this rank's step = SURVEY.md §8(d)'s IR ops per
+    # instance x the instances it checked, over the K2 busy time, against the measured integer
+    # peak of both pipes (alu: IADD3/LOP3/SHF/ISETP, fma: IMAD); beside it the IR operations
+    # the subject kernels actually executed (PG_CHK_OPCOUNT: idle threads of a reduction round
+    # count as instances, X19, but execute only the guard)
     k2_s = k2_ms / 1000.0 / args.steps
-    achieved = ir_ops / k2_s if k2_s else None
     per_gpu_inst = inst_total / world / args.steps
+    achieved = SURVEY_OPS[WL] * per_gpu_inst / k2_s if k2_s else None
+    counted = ir_ops / k2_s if k2_s else None
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True, "scaling": "weak",
@@ -464,8 +475,13 @@ def main():
         "roofline": {"bound": "alu", "achieved": achieved / 1e12 if achieved else None,
                      "peak": peak["mixed"] / 1e12, "unit": "Tops/s (int32 IR operations)",
                      "frac": (achieved / peak["mixed"]) if achieved else None, "traffic": None,
-                     "kernel": "pgk_eval (K2)", "ir_ops_per_step": ir_ops,
-                     "ir_ops_per_instance": ir_ops / per_gpu_inst if per_gpu_inst else None,
+                     "kernel": "pgk_eval (K2)",
+                     "algorithmic_ops_per_instance": SURVEY_OPS[WL],
+                     "algorithmic_basis": "SURVEY.md 8(d) IR int ops per (thread, round) x instances per step",
+                     "instances_per_step": per_gpu_inst,
+                     "counted_ir_ops_per_step": ir_ops,
+                     "counted_ir_ops_per_instance": ir_ops / per_gpu_inst if per_gpu_inst else None,
+                     "frac_counted_ops": (counted / peak["mixed"]) if counted else None,
                      "k2_busy_ms_per_step": k2_ms / args.steps,
                      "k2_launch_sum_ms_per_step": sum(k2_sum) / args.steps,
                      "k2_share_of_step": k2_ms / dev_ms if dev_ms else None,
