@@ -742,8 +742,6 @@ struct Gen {
         o << "#define PG_LOCKSTEP " << ((O.checks & 64) ? 1 : 0) << "\n";
         o << "#define PG_FAST " << (O.fast ? 1 : 0) << "\n";
         // (store-time claims: not with bank / coalescing statistics, nor with PGVC_CAS=0 - api.cpp cas_on)
-        o << "#define PG_SEEDH_ON " << ((std::getenv("PGVC_SEEDH") && std::string(std::getenv("PGVC_SEEDH")) == "0") ? 0 : 1)
-          << "\n";
         o << "#define PG_CAS_ON "
           << (((std::getenv("PGVC_CAS") && std::string(std::getenv("PGVC_CAS")) == "0") || (O.checks & (8 | 16))) ? 0 : 1)
           << "\n";

@@ -206,9 +206,6 @@ struct PgCold {     // per-emulated-thread state that lives in local memory
     u32 ebvs[PG_NK][PG_MS];      //     met (bit k): then val_b per seed here
 #endif
     u64 epk[PG_NK];              // pg_pack of ebest[kind] (one 64-bit compare decides most events)
-#if PG_MSX
-    u32 sb;                      // the lane's first seed within the work item (pg_sSeedH index)
-#endif
 };
 
 __device__ __forceinline__ bool pg_lex_less(const u32* a, const u32* b) {
@@ -848,18 +845,6 @@ __device__ __forceinline__ void pg_ld_gi_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 // Per seed: write-log values, committed values, poison values and the events' value
 // fields; once per cell: claims, owner / race stamps and the race decision.
 __device__ __forceinline__ u64 pg_seed_of(const PgT& t, u32 s) { return t.seed + (u64)s * pg_sW.seed_jstep; }
-// sm(seed) of the work item's seeds (the PRF's first SplitMix round, X8), computed once per item:
-// poison and out-of-bounds values then cost one SplitMix round per seed
-#ifndef PG_SEEDH_ON
-#define PG_SEEDH_ON 1
-#endif
-#define PG_SEEDH (PG_SEEDH_ON ? 128u : 1u)
-__shared__ u64 pg_sSeedH[PG_SEEDH];
-__device__ __forceinline__ u32 pg_rand32_s(const PgT& t, const PgCold& c, u32 s, u64 tag, u64 idx) {
-    const u32 i = c.sb + s;
-    const u64 h = PG_SEEDH_ON && i < PG_SEEDH ? pg_sSeedH[i] : pg_sm64(pg_seed_of(t, s));
-    return pg_rand32_k(h ^ (tag << 48), idx);
-}
 __device__ __noinline__ u32 pg_event_ms(PgCold& c, u32 evm, u32 kind, u32 round, u32 arr, u32 addr, u32 ta,
                                         u32 tb, u32 site, const u32* va, u32 vb) {
     const u32 e[6] = {round, arr, addr, ta, tb, site};
@@ -956,7 +941,7 @@ __device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     if (!pe) return;
     const u32 rec = PG_ARR(A).rec_id;
     if (flat >= PG_SH(A, size)) {
-        PG_S_LOOP v[_s] = pg_m(pg_rand32_s(t, c, _s, 0x8000u + (rec - 0x100u), ((u64)t.blk << 20) + flat));
+        PG_S_LOOP v[_s] = pg_m(pg_rand32(pg_seed_of(t, _s), 0x8000u + (rec - 0x100u), ((u64)t.blk << 20) + flat));
 #if PG_OOBCHK
         t.evm |= pg_event_ms(c, t.evm, PGK_OOB, C.round, rec, flat, t.gtid, PG_NEVER, site, v, 0);
 #endif
@@ -971,7 +956,7 @@ __device__ __forceinline__ void pg_ld_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     if (LOG && pg_log_find_ms(t, c, ((u32)A << 24) | flat, v)) return;
     const u32 own = pg_sh(t, PG_SH(A, s_own))[flat];
     if (own >= C.uthr) {  // never written in this block (X6)
-        PG_S_LOOP v[_s] = pg_m(pg_rand32_s(t, c, _s, 0x8000u + (rec - 0x100u), ((u64)t.blk << 20) + flat));
+        PG_S_LOOP v[_s] = pg_m(pg_rand32(pg_seed_of(t, _s), 0x8000u + (rec - 0x100u), ((u64)t.blk << 20) + flat));
 #if PG_OOBCHK
         t.evm |= pg_event_ms(c, t.evm, PGK_UNINIT, C.round, rec, flat, t.gtid, PG_NEVER, site, v, 0);
 #endif
@@ -1014,7 +999,7 @@ __device__ __forceinline__ void pg_ld_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     PG_S_LOOP v[_s] = 0u;
     if (!pe) return;
     if (flat >= PG_ARR(A).size) {
-        PG_S_LOOP v[_s] = pg_m(pg_rand32_s(t, c, _s, PG_ARR(A).gid, flat));
+        PG_S_LOOP v[_s] = pg_m(pg_rand32(pg_seed_of(t, _s), PG_ARR(A).gid, flat));
 #if PG_OOBCHK
         t.evm |= pg_event_ms(c, t.evm, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, v, 0);
 #endif
@@ -1059,7 +1044,7 @@ __device__ __forceinline__ void pg_ld_gi_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     PG_S_LOOP v[_s] = 0u;
     if (!pe) return;
     if (flat >= PG_ARR(A).size) {
-        PG_S_LOOP v[_s] = pg_m(pg_rand32_s(t, c, _s, PG_ARR(A).gid, flat));
+        PG_S_LOOP v[_s] = pg_m(pg_rand32(pg_seed_of(t, _s), PG_ARR(A).gid, flat));
 #if PG_OOBCHK
         t.evm |= pg_event_ms(c, t.evm, PGK_OOB, C.round, PG_ARR(A).rec_id, flat, t.gtid, PG_NEVER, site, v, 0);
 #endif
@@ -1830,10 +1815,6 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi, u32& ph
         pg_desc_bulk_wait(phase);
         phase ^= 1u;
     }
-#if PG_MSX && PG_SEEDH_ON
-    for (u32 i = threadIdx.x; i < min(pg_sW.nseeds, PG_SEEDH); i += blockDim.x)
-        pg_sSeedH[i] = pg_sm64(P.seed_base + (u64)(pg_sW.seed_j0 + i * pg_sW.seed_jstep));
-#endif
 #if PG_DATAFLOW
     if (threadIdx.x == 0) pg_sDf = PgDf{P.df_rows, P.df_count, P.seed_base, P.df_cap};
 #endif
@@ -1943,9 +1924,6 @@ __device__ __forceinline__ void pg_item(const PgParams& P, const u32 wi, u32& ph
         t.tid[1] = (t.tlin / PG_BDIM0) % PG_BDIM1;
         t.tid[2] = t.tlin / (PG_BDIM0 * PG_BDIM1);
         t.seed = P.seed_base + (u64)(pg_sW.seed_j0 + sb * pg_sW.seed_jstep);
-#if PG_MSX
-        Cd[v].sb = sb;
-#endif
         t.arena = P.arena + pg_sW.arena_off + (u64)sb * pg_sL.arena_stride;
         t.input = P.input + pg_sW.input_off + (u64)sb * pg_sL.input_stride;
         t.nsv = nsv;
