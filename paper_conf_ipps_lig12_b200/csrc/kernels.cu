@@ -121,15 +121,16 @@ __device__ __forceinline__ void pg_cmp_rows(const PgCmp& c, const PgRegions& R, 
         w.size[m] = on ? c.size[m] : 0u;
     }
 }
-__device__ __forceinline__ void pg_cmp_cell(const PgCmpRows& w, u32 i, u32 (&cnt)[PG_MAXK], u32 (&mn)[PG_MAXK]) {
-    u32 v[PG_MAXK];
+// one cell i: the members' values, then for each member a the mismatching pairs (a, b > a)
+// (NM: members of the job - specialised, so a 2-kernel check does one pair, not 28)
+template <u32 NM>
+__device__ __forceinline__ void pg_cmp_vals(const PgCmpRows& w, u32 i, const u32 (&v)[PG_MAXK], u32 (&cnt)[PG_MAXK],
+                                            u32 (&mn)[PG_MAXK]) {
 #pragma unroll
-    for (u32 m = 0; m < PG_MAXK; m++) v[m] = i < w.size[m] ? w.p[m][i] : 0u;
-#pragma unroll
-    for (u32 a = 0; a + 1 < PG_MAXK; a++) {
+    for (u32 a = 0; a + 1 < NM; a++) {
         u32 k = 0;
 #pragma unroll
-        for (u32 b = a + 1; b < PG_MAXK; b++)
+        for (u32 b = a + 1; b < NM; b++)
             k += (v[a] != v[b]) & (u32)((w.mask >> (a * PG_MAXK + b)) & 1ull) & (i < w.size[a]) & (i < w.size[b]);
         if (k) {
             cnt[a] += k;
@@ -137,7 +138,85 @@ __device__ __forceinline__ void pg_cmp_cell(const PgCmpRows& w, u32 i, u32 (&cnt
         }
     }
 }
-__global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs, u32 n_jobs, u32 n_tasks,
+template <u32 NM>
+__device__ __forceinline__ void pg_cmp_cell(const PgCmpRows& w, u32 i, u32 (&cnt)[PG_MAXK], u32 (&mn)[PG_MAXK]) {
+    u32 v[PG_MAXK];
+#pragma unroll
+    for (u32 m = 0; m < NM; m++) v[m] = i < w.size[m] ? w.p[m][i] : 0u;
+    pg_cmp_vals<NM>(w, i, v, cnt, mn);
+}
+// four consecutive cells q..q+3 (q a multiple of 4, rows 16-byte aligned): one 128-bit load
+// per member, then the cells in index order
+template <u32 NM>
+__device__ __forceinline__ void pg_cmp_cell4(const PgCmpRows& w, u32 q, u32 (&cnt)[PG_MAXK], u32 (&mn)[PG_MAXK]) {
+    uint4 v4[NM];
+#pragma unroll
+    for (u32 m = 0; m < NM; m++) {
+        if (q + 4u <= w.size[m]) {
+            v4[m] = __ldcs((const uint4*)(w.p[m] + q));
+        } else {
+            v4[m].x = q < w.size[m] ? w.p[m][q] : 0u;
+            v4[m].y = q + 1u < w.size[m] ? w.p[m][q + 1u] : 0u;
+            v4[m].z = q + 2u < w.size[m] ? w.p[m][q + 2u] : 0u;
+            v4[m].w = 0u;
+        }
+    }
+#pragma unroll
+    for (u32 e = 0; e < 4u; e++) {
+        u32 v[PG_MAXK];
+#pragma unroll
+        for (u32 m = 0; m < NM; m++) v[m] = e == 0 ? v4[m].x : e == 1 ? v4[m].y : e == 2 ? v4[m].z : v4[m].w;
+        pg_cmp_vals<NM>(w, q + e, v, cnt, mn);
+    }
+}
+// cells [lo, hi) of one instance by `lanes` threads: 128-bit streaming loads, 4 cells per
+// thread per step, several steps in flight (rows are 128-byte aligned in the arenas; checked,
+// the scalar loop otherwise)
+template <u32 NM>
+__device__ __forceinline__ void pg_cmp_range(const PgCmpRows& w, u32 lo, u32 hi, u32 lane, u32 lanes,
+                                             u32 (&cnt)[PG_MAXK], u32 (&mn)[PG_MAXK]) {
+    u32 al = 0;
+#pragma unroll
+    for (u32 m = 0; m < NM; m++) al |= (u32)(uintptr_t)w.p[m];
+    if ((al & 15u) == 0u && (lo & 3u) == 0u) {
+        // U steps per trip: their loads issue together (fewer for many members: registers)
+        constexpr u32 U = NM <= 2 ? 4u : NM <= 4 ? 2u : 1u;
+        const u32 st = 4u * lanes;
+        u32 q = lo + 4u * lane;
+        for (; q + (U - 1u) * st + 4u <= hi; q += U * st) {
+#pragma unroll
+            for (u32 u = 0; u < U; u++) pg_cmp_cell4<NM>(w, q + u * st, cnt, mn);
+        }
+        for (; q < hi; q += st) {
+            if (q + 4u <= hi) pg_cmp_cell4<NM>(w, q, cnt, mn);
+            else
+                for (u32 i = q; i < hi; i++) pg_cmp_cell<NM>(w, i, cnt, mn);
+        }
+    } else {
+        for (u32 i = lo + lane; i < hi; i += lanes) pg_cmp_cell<NM>(w, i, cnt, mn);
+    }
+}
+template <u32 NMX>
+__device__ __forceinline__ void pg_cmp_any(const PgCmpRows& w, u32 nm, u32 lo, u32 hi, u32 lane, u32 lanes,
+                                           u32 (&cnt)[PG_MAXK], u32 (&mn)[PG_MAXK]) {
+    if (NMX <= 2u) {   // (pairs: the kernel instance of the 2-member checks)
+        pg_cmp_range<2>(w, lo, hi, lane, lanes, cnt, mn);
+        return;
+    }
+    switch (nm) {
+        case 0: case 1: case 2: pg_cmp_range<2>(w, lo, hi, lane, lanes, cnt, mn); break;
+        case 3: pg_cmp_range<3>(w, lo, hi, lane, lanes, cnt, mn); break;
+        case 4: pg_cmp_range<4>(w, lo, hi, lane, lanes, cnt, mn); break;
+        case 5: pg_cmp_range<5>(w, lo, hi, lane, lanes, cnt, mn); break;
+        case 6: pg_cmp_range<6>(w, lo, hi, lane, lanes, cnt, mn); break;
+        case 7: pg_cmp_range<7>(w, lo, hi, lane, lanes, cnt, mn); break;
+        default: pg_cmp_range<PG_MAXK>(w, lo, hi, lane, lanes, cnt, mn); break;
+    }
+}
+// NMX: the most members of any job of the launch (2: pairs - 4 CTAs per SM within the
+// register budget; PG_MAXK: N-kernel checks)
+template <u32 NMX>
+__global__ void __launch_bounds__(256, NMX <= 2 ? 4 : 2) pg_compare(const PgCmp* __restrict__ jobs, u32 n_jobs, u32 n_tasks,
                                                   const PgRegions R, PgSlot* slots, u64* mm_key) {
     __shared__ u32 s_cnt[PG_MAXK], s_min[PG_MAXK];
     __shared__ u32 s_job;
@@ -153,7 +232,7 @@ __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs
             if (inst >= c.n_inst) continue;
             PgCmpRows w;
             pg_cmp_rows(c, R, inst, w);
-            for (u32 i = lane; i < c.n; i += 32u) pg_cmp_cell(w, i, cnt, mn);
+            pg_cmp_any<NMX>(w, c.nm, 0u, c.n, lane, 32u, cnt, mn);
 #pragma unroll
             for (u32 a = 0; a + 1 < PG_MAXK; a++) {
                 if (a + 1 >= c.nm) break;
@@ -172,7 +251,7 @@ __global__ void __launch_bounds__(256) pg_compare(const PgCmp* __restrict__ jobs
         __syncthreads();
         PgCmpRows w;
         pg_cmp_rows(c, R, inst, w);
-        for (u32 i = w0 + threadIdx.x; i < w1; i += blockDim.x) pg_cmp_cell(w, i, cnt, mn);
+        pg_cmp_any<NMX>(w, c.nm, w0, w1, threadIdx.x, blockDim.x, cnt, mn);
 #pragma unroll
         for (u32 a = 0; a + 1 < PG_MAXK; a++) {
             if (a + 1 >= c.nm) break;
@@ -681,10 +760,11 @@ cudaError_t count_reduce(const u64* inst_cnt, u32 n, long long* counts, cudaStre
     return cudaGetLastError();
 }
 
-cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 n_tasks, u32 max_inst, const PgRegions& R, PgSlot* slots,
-                    u64* mm_key, u64* mm2, cudaStream_t st) {
+cudaError_t compare(const PgCmp* jobs, u32 n_jobs, u32 n_tasks, u32 max_nm, u32 max_inst, const PgRegions& R,
+                    PgSlot* slots, u64* mm_key, u64* mm2, cudaStream_t st) {
     if (!n_jobs) return cudaSuccess;
-    pg_compare<<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, R, slots, mm_key);
+    if (max_nm <= 2u) pg_compare<2><<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, R, slots, mm_key);
+    else pg_compare<PG_MAXK><<<task_grid(n_tasks), 256, 0, st>>>(jobs, n_jobs, n_tasks, R, slots, mm_key);
     for (u32 j0 = 0; j0 < n_jobs; j0 += 65535u) {
         const u32 nj = n_jobs - j0 < 65535u ? n_jobs - j0 : 65535u;
         dim3 g2((max_inst + 127) / 128, nj);
