@@ -433,6 +433,27 @@ __device__ __forceinline__ u32 pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell,
     return 0u;
 }
 
+// Stamps of a global array the kernel writes: in the instance arena, or - single-block
+// launches (PgArr flags bit 1, PgSA::gsh) - in the group's shared region, where they cost
+// shared-memory atomics instead of L2 atomics (no other block can touch the cells)
+#ifdef PG_S_T
+#define PG_GSH(A) ((u32)PgSA<A>::gsh)
+#else
+#define PG_GSH(A) ((pg_sL.arr[A].flags >> 1) & 1u)
+#endif
+template <int A> __device__ __forceinline__ u32* pg_gown(const PgT& t) {
+    return PG_GSH(A) ? pg_sh(t, PG_SH(A, s_own)) : t.arena + PG_ARR(A).off_own;
+}
+template <int A> __device__ __forceinline__ u32* pg_gwmax(const PgT& t) {
+    return PG_GSH(A) ? pg_sh(t, PG_SH(A, s_wmax)) : t.arena + PG_ARR(A).off_wmax;
+}
+template <int A> __device__ __forceinline__ u32* pg_grmin(const PgT& t) {
+    return PG_GSH(A) ? pg_sh(t, PG_SH(A, s_rmin)) : t.arena + PG_ARR(A).off_rmin;
+}
+template <int A> __device__ __forceinline__ u32* pg_grmax(const PgT& t) {
+    return PG_GSH(A) ? pg_sh(t, PG_SH(A, s_rmax)) : t.arena + PG_ARR(A).off_rmax;
+}
+
 // Claim (exact protocol): atomicMin on the cell's claim stamp (newest round wins over stale
 // stamps, the min tid wins within the round) plus atomicMax for WW detection.  Shared arrays
 // claim into s_clm when claims happen at store time (PG_CAS: s_own keeps the committed owner
@@ -447,9 +468,9 @@ __device__ __forceinline__ void pg_claim_sh(const PgC& C, const PgT& t, u32 flat
 }
 template <int A>
 __device__ __forceinline__ void pg_claim_gt(const PgC& C, const PgT& t, u32 flat) {
-    atomicMin(t.arena + PG_ARR(A).off_own + flat, pg_stamp_min(C, t));
+    atomicMin(pg_gown<A>(t) + flat, pg_stamp_min(C, t));
 #if PG_RACECHK
-    if (PG_T > 1u) atomicMax(t.arena + PG_ARR(A).off_wmax + flat, pg_stamp_max(C, t));
+    if (PG_T > 1u) atomicMax(pg_gwmax<A>(t) + flat, pg_stamp_max(C, t));
 #endif
 }
 
@@ -661,7 +682,7 @@ __device__ __forceinline__ void pg_fcheck_sh(const PgC& C, PgT& t, u32 flat) {
 template <int A>
 __device__ __forceinline__ void pg_fcheck_gt(const PgC& C, PgT& t, u32 flat) {
     const u64 so = (u64)C.par * PG_ARR(A).size + flat;
-    t.fl |= pg_fast_rw(C, t, t.arena[PG_ARR(A).off_rmin + so], t.arena[PG_ARR(A).off_rmax + so]);
+    t.fl |= pg_fast_rw(C, t, pg_grmin<A>(t)[so], pg_grmax<A>(t)[so]);
 }
 // (C still describes the round just finished)
 template <class K>
@@ -798,7 +819,7 @@ __device__ __forceinline__ void pg_ld_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     pg_xb_mark_ms<A>(t, flat);
     if (RD && PG_T > 1u) {
         const u64 so = (u64)C.par * PG_ARR(A).size + flat;
-        pg_fread(t.arena + PG_ARR(A).off_rmin + so, t.arena + PG_ARR(A).off_rmax + so, C.smax, t.tlin);
+        pg_fread(pg_grmin<A>(t) + so, pg_grmax<A>(t) + so, C.smax, t.tlin);
     }
     const u64 st = pg_sL.arena_stride;
     PG_S_LOOP if (_s < t.nsv) v[_s] = t.arena[_s * st + PG_ARR(A).off_val + flat];
@@ -812,7 +833,7 @@ __device__ __forceinline__ void pg_st_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
         return;
     }
     pg_xb_mark_ms<A>(t, flat);
-    u32* own = t.arena + PG_ARR(A).off_own + flat;
+    u32* own = pg_gown<A>(t) + flat;
     const u32 me = C.smin | t.tlin;
     if (PG_T > 1u) {
         const u32 old = atomicMin(own, me);
@@ -1008,8 +1029,8 @@ __device__ __forceinline__ void pg_ld_gt_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     pg_xb_mark_ms<A>(t, flat);
 #if PG_RACECHK
     if (RD && PG_T > 1u) {
-        atomicMin(t.arena + PG_ARR(A).off_rmin + flat, pg_stamp_min(C, t));
-        atomicMax(t.arena + PG_ARR(A).off_rmax + flat, pg_stamp_max(C, t));
+        atomicMin(pg_grmin<A>(t) + flat, pg_stamp_min(C, t));
+        atomicMax(pg_grmax<A>(t) + flat, pg_stamp_max(C, t));
     }
 #endif
     if (LOG && pg_log_find_ms(t, c, ((u32)A << 24) | flat, v)) return;
@@ -1104,7 +1125,7 @@ template <int A, bool RD>
 __device__ __forceinline__ void pg_check_gt_ms(const PgC& C, PgT& t, PgCold& c, u32 flat, const u32* val, u32 site) {
     const u64 st = pg_sL.arena_stride;
     if (PG_T == 1u) {
-        t.arena[PG_ARR(A).off_own + flat] = pg_stamp_min(C, t);
+        pg_gown<A>(t)[flat] = pg_stamp_min(C, t);
         PG_S_LOOP {
             if (_s < t.nsv) {
                 t.arena[_s * st + PG_ARR(A).off_val + flat] = val[_s];
@@ -1113,7 +1134,7 @@ __device__ __forceinline__ void pg_check_gt_ms(const PgC& C, PgT& t, PgCold& c, 
         }
         return;
     }
-    const u32 own = t.arena[PG_ARR(A).off_own + flat];
+    const u32 own = pg_gown<A>(t)[flat];
     if (own == pg_stamp_min(C, t)) {
         PG_S_LOOP {
             if (_s < t.nsv) {
@@ -1124,9 +1145,9 @@ __device__ __forceinline__ void pg_check_gt_ms(const PgC& C, PgT& t, PgCold& c, 
     }
 #if PG_RACECHK
     if (PG_T > 1u) {
-        const u32 wmax = t.arena[PG_ARR(A).off_wmax + flat];
-        const u32 rmin = RD ? t.arena[PG_ARR(A).off_rmin + flat] : 0u;
-        const u32 rmax = RD ? t.arena[PG_ARR(A).off_rmax + flat] : 0u;
+        const u32 wmax = pg_gwmax<A>(t)[flat];
+        const u32 rmin = RD ? pg_grmin<A>(t)[flat] : 0u;
+        const u32 rmax = RD ? pg_grmax<A>(t)[flat] : 0u;
         if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
             (RD && (rmax >> 12) == C.step && (((rmin ^ own) | (rmax ^ own)) & 0xFFFu)))
             t.evm = pg_race_check_ms(C.round, C.step, t.tlin, t.gtid, c, t.evm, val, site, PG_ARR(A).rec_id, flat,
@@ -1167,14 +1188,14 @@ __device__ __forceinline__ u32 pg_ld_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32 
 #if PG_FAST
     if (RD && PG_T > 1u) {
         const u64 so = (u64)C.par * PG_ARR(A).size + flat;
-        pg_fread(t.arena + PG_ARR(A).off_rmin + so, t.arena + PG_ARR(A).off_rmax + so, C.smax, t.tlin);
+        pg_fread(pg_grmin<A>(t) + so, pg_grmax<A>(t) + so, C.smax, t.tlin);
     }
     return t.arena[PG_ARR(A).off_val + flat];
 #else
 #if PG_RACECHK
     if (RD && PG_T > 1u) {
-        atomicMin(t.arena + PG_ARR(A).off_rmin + flat, pg_stamp_min(C, t));
-        atomicMax(t.arena + PG_ARR(A).off_rmax + flat, pg_stamp_max(C, t));
+        atomicMin(pg_grmin<A>(t) + flat, pg_stamp_min(C, t));
+        atomicMax(pg_grmax<A>(t) + flat, pg_stamp_max(C, t));
     }
 #endif
     u32 v;
@@ -1208,7 +1229,7 @@ __device__ __forceinline__ void pg_st_gt(PgC& C, PgT& t, PgCold& c, u64* ss, u32
     pg_xb_mark<A>(t, flat);
 #if PG_FAST
     {
-        u32* own = t.arena + PG_ARR(A).off_own + flat;
+        u32* own = pg_gown<A>(t) + flat;
         const u32 me = C.smin | t.tlin;
         if (PG_T > 1u) {
             const u32 old = atomicMin(own, me);
@@ -1321,21 +1342,21 @@ __device__ __forceinline__ void pg_check_sh(const PgC& C, PgT& t, PgCold& c, u32
 template <int A, bool RD>
 __device__ __forceinline__ void pg_check_gt(const PgC& C, PgT& t, PgCold& c, u32 flat, u32 val, u32 site) {
     if (PG_T == 1u) {
-        t.arena[PG_ARR(A).off_own + flat] = pg_stamp_min(C, t);
+        pg_gown<A>(t)[flat] = pg_stamp_min(C, t);
         t.arena[PG_ARR(A).off_val + flat] = val;
         t.arena[PG_ARR(A).off_lw + flat] = t.gtid + 1u;
         return;
     }
-    const u32 own = t.arena[PG_ARR(A).off_own + flat];
+    const u32 own = pg_gown<A>(t)[flat];
     if (own == pg_stamp_min(C, t)) {
         t.arena[PG_ARR(A).off_val + flat] = val;
         t.arena[PG_ARR(A).off_lw + flat] = t.gtid + 1u;
     }
 #if PG_RACECHK
     if (PG_T > 1u) {
-        const u32 wmax = t.arena[PG_ARR(A).off_wmax + flat];
-        const u32 rmin = RD ? t.arena[PG_ARR(A).off_rmin + flat] : 0u;
-        const u32 rmax = RD ? t.arena[PG_ARR(A).off_rmax + flat] : 0u;
+        const u32 wmax = pg_gwmax<A>(t)[flat];
+        const u32 rmin = RD ? pg_grmin<A>(t)[flat] : 0u;
+        const u32 rmax = RD ? pg_grmax<A>(t)[flat] : 0u;
         // (a cell only its writer read this round is no RW race: skip the slow path)
         if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
             (RD && (rmax >> 12) == C.step && (((rmin ^ own) | (rmax ^ own)) & 0xFFFu)))

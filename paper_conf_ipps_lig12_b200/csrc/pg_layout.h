@@ -34,8 +34,10 @@ struct PgArr {
     u32 kind;       // PGA_*
     u32 rec_id;     // array id in records: gid | 0x100 + slot | 0x200 + slot
     u32 gid;        // pair-level global id (PRF tag, X8)
-    u32 flags;      // bit0: reader stamps present (array read and written, race checks on)
-    // shared arrays: byte offsets in the group's shared region
+    u32 flags;      // bit0: reader stamps present (array read and written, race checks on);
+                    // bit1: a global array whose stamps live in shared memory (single-block launch)
+    // shared arrays (and the stamps of flags-bit-1 global arrays): byte offsets in the group's
+    // shared region
     u32 s_val, s_own, s_wmax, s_rmin, s_rmax;
     u32 s_clm;      // claims of the round (exact protocol with claims at store time; s_own then
                     // holds the committed owner only, which loads of the same round consult)
