@@ -742,6 +742,8 @@ struct Gen {
         o << "#define PG_LOCKSTEP " << ((O.checks & 64) ? 1 : 0) << "\n";
         o << "#define PG_FAST " << (O.fast ? 1 : 0) << "\n";
         // (store-time claims: not with bank / coalescing statistics, nor with PGVC_CAS=0 - api.cpp cas_on)
+        if (std::getenv("PGVC_RC_INLINE") && std::string(std::getenv("PGVC_RC_INLINE")) == "1")
+            o << "#define PG_RC_INLINE __forceinline__\n";
         o << "#define PG_CAS_ON "
           << (((std::getenv("PGVC_CAS") && std::string(std::getenv("PGVC_CAS")) == "0") || (O.checks & (8 | 16))) ? 0 : 1)
           << "\n";

@@ -46,6 +46,10 @@
 #ifndef PG_CAS_ON
 #define PG_CAS_ON 1    // (PGVC_CAS=0: claims in their own phase, diagnostics)
 #endif
+// the round-end race decision of a racy cell (cold: one thread per racy cell and round)
+#ifndef PG_RC_INLINE
+#define PG_RC_INLINE __noinline__
+#endif
 #define PG_CAS (PG_CAS_ON && !PG_FAST && !PG_DATAFLOW && !PG_VCLIT && !PG_DIVBAR && !PG_LOCKSTEP)
 #define PG_MSX (PG_MS > 1 && !PG_FAST)
 #define PG_S_LOOP _Pragma("unroll") for (u32 _s = 0; _s < (u32)PG_MS; _s++)
@@ -1077,7 +1081,7 @@ __device__ __forceinline__ void pg_ld_gi_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 }
 // round end of the exact protocol: the owner commits every seed's value; race decisions
 // are per cell, their records carry each seed's value
-__device__ __noinline__ u32 pg_race_check_ms(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 evm,
+__device__ PG_RC_INLINE u32 pg_race_check_ms(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 evm,
                                              const u32* val, u32 site, u32 rec, u32 flat, u32 own, u32 wmax,
                                              u32 has_readers, u32 rmin, u32 rmax) {
     const u32 base = gtid - tlin;
@@ -1294,7 +1298,7 @@ __device__ __forceinline__ void pg_tick(PgC& C, PgT& t, PgCold& c, u32 act) {
 // its value (and, for global arrays, itself as last writer); with race checks
 // the owner reports WW, and the thread the X16 rule names tid_a reports RW.
 
-__device__ __noinline__ u32 pg_race_check(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 evm, u32 val,
+__device__ PG_RC_INLINE u32 pg_race_check(u32 round, u32 step, u32 tlin, u32 gtid, PgCold& c, u32 evm, u32 val,
                                           u32 site, u32 rec, u32 flat, u32 own, u32 wmax, u32 has_readers, u32 rmin,
                                           u32 rmax) {
     const u32 base = gtid - tlin;

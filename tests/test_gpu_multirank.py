@@ -97,6 +97,25 @@ def test_bench_world2_branch_matches_world1(env):  # noqa: F811
     # 2 ranks x 4 seeds (seeds r, r+2, ...) = the 1-rank run's 8 seeds: same H9-reduced summary
     assert two["check"] == one["check"]
     assert two["value"] > 0 and two["e2e"]["value"] > 0
+    for line in (one, two):
+        _bench_contract(line)
+
+
+def _bench_contract(d):
+    # the JSON line's measurement contract: the roofline follows from its own fields
+    # (SURVEY.md 8(d)'s per-unit work x the instances of a step / the K2 busy time)
+    r = d["roofline"]
+    assert r["bound"] == "alu" and r["unit"].startswith("Tops/s")
+    per_gpu = d["check"]["instances"] / d["n_gpus"]
+    assert abs(r["instances_per_step"] - per_gpu) <= 1e-6 * per_gpu
+    achieved = r["algorithmic_ops_per_instance"] * r["instances_per_step"] / (r["k2_busy_ms_per_step"] / 1e3)
+    assert abs(r["achieved"] * 1e12 - achieved) <= 1e-6 * achieved
+    assert abs(r["frac"] - r["achieved"] / r["peak"]) <= 1e-9
+    assert 0 < r["frac"] < 1 and 0 < r["frac_counted_ops"] < r["frac"]
+    assert r["k2_busy_ms_per_step"] <= d["ms_per_step"] * 1.0001
+    assert d["gpu_launches"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
+    assert d["step_ms"]["min"] <= d["step_ms"]["median"] <= d["step_ms"]["max"]
+    assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
 
 
 @pytest.mark.timeout(900)
