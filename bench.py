@@ -458,10 +458,12 @@ def main():
     e2e = inst_total / wall_s
     sm_max = clk.get("sm_max_mhz") or measured_peaks().get("sm_max_mhz", 1965.0)
     # roofline (per GPU): algorithmic work of this rank's step = SURVEY.md §8(d)'s IR ops per
-    # instance x the instances it checked, over the K2 busy time, against the measured integer
-    # peak of both pipes (alu: IADD3/LOP3/SHF/ISETP, fma: IMAD); beside it the IR operations
-    # the subject kernels actually executed (PG_CHK_OPCOUNT: idle threads of a reduction round
-    # count as instances, X19, but execute only the guard)
+    # instance x the instances it checked, over the K2 busy time, against SURVEY.md §8(d)'s
+    # denominator, the INT32 ALU-pipe peak (148 SMs x 64 lanes/clk x f: IADD3/LOP3/SHF/ISETP,
+    # the pipe the IR's adds, logic, shifts and compares issue to), measured live; beside it
+    # the fraction of both integer pipes (alu + fma/IMAD: the hard upper bound) and the IR
+    # operations the subject kernels actually executed (PG_CHK_OPCOUNT: idle threads of a
+    # reduction round count as instances, X19, but execute only the guard)
     k2_s = k2_ms / 1000.0 / args.steps
     per_gpu_inst = inst_total / world / args.steps
     achieved = SURVEY_OPS[WL] * per_gpu_inst / k2_s if k2_s else None
@@ -473,21 +475,22 @@ def main():
         "config": {"workload": workload_desc(), "seeds_per_gpu": SEEDS_PER_GPU, "l2": "flushed before every step",
                    "streams": len(side), "parallelism": "dp%d over seeds" % world},
         "roofline": {"bound": "alu", "achieved": achieved / 1e12 if achieved else None,
-                     "peak": peak["mixed"] / 1e12, "unit": "Tops/s (int32 IR operations)",
-                     "frac": (achieved / peak["mixed"]) if achieved else None, "traffic": None,
+                     "peak": peak["alu"] / 1e12, "unit": "Tops/s (int32 IR operations)",
+                     "frac": (achieved / peak["alu"]) if achieved else None, "traffic": None,
                      "kernel": "pgk_eval (K2)",
                      "algorithmic_ops_per_instance": SURVEY_OPS[WL],
                      "algorithmic_basis": "SURVEY.md 8(d) IR int ops per (thread, round) x instances per step",
                      "instances_per_step": per_gpu_inst,
                      "counted_ir_ops_per_step": ir_ops,
                      "counted_ir_ops_per_instance": ir_ops / per_gpu_inst if per_gpu_inst else None,
-                     "frac_counted_ops": (counted / peak["mixed"]) if counted else None,
+                     "frac_counted_ops": (counted / peak["alu"]) if counted else None,
                      "k2_busy_ms_per_step": k2_ms / args.steps,
                      "k2_launch_sum_ms_per_step": sum(k2_sum) / args.steps,
                      "k2_share_of_step": k2_ms / dev_ms if dev_ms else None,
-                     "peak_source": "measured live: pg_measure_int32_peak, LOP3 + IMAD chains on both pipes",
-                     "peak_alu_pipe": peak["alu"] / 1e12, "peak_fma_pipe": peak["fma"] / 1e12,
-                     "frac_of_alu_pipe": (achieved / peak["alu"]) if achieved else None,
+                     "peak_source": "measured live: pg_measure_int32_peak, LOP3 chains on the alu pipe "
+                                    "(SURVEY.md 8(d): 148 SMs x 64 lanes/clk x f)",
+                     "peak_both_pipes": peak["mixed"] / 1e12, "peak_fma_pipe": peak["fma"] / 1e12,
+                     "frac_of_both_pipes": (achieved / peak["mixed"]) if achieved else None,
                      "time_basis": "union of K2 launch intervals (CUDA events in the check graphs)"},
         "e2e": {"value": e2e, "unit": UNIT, "h2d_bytes_per_step": h2d // args.steps,
                 "d2h_bytes_per_step": d2h // args.steps},

@@ -231,6 +231,12 @@ int pg_ir_info(const pg_ir *k, uint32_t *n_sites, uint32_t *n_globals, uint32_t 
  * compare-exchange, whose store guard depends on the data).  *n_tainted = the variables
  * that may hold an input-dependent value.  PG_E_ARG on a null kernel. */
 int pg_ir_seed_oblivious(const pg_ir *k, uint32_t *oblivious, uint32_t *n_tainted);
+/* *block_private = 1 when every global array the kernel writes is never loaded and every
+ * store to it has the flat index bid.x: distinct blocks of a one-dimensional grid then
+ * write distinct cells and read none another block writes, so the cross-block race X4 (XB)
+ * cannot occur and checks of such launches skip the XB stamps, K2b and the sequential pass
+ * (the SDK reductions' g_odata[bid.x]).  PG_E_ARG on a null kernel. */
+int pg_ir_block_private(const pg_ir *k, uint32_t *block_private);
 /* Generated CUDA source of the evaluation kernel for (bits, checks, bank_model). */
 int pg_ir_source(const pg_ir *k, uint32_t bits, uint32_t checks, uint32_t bank_model, char *buf, size_t cap,
                  size_t *len);

@@ -852,6 +852,25 @@ bool seed_oblivious(const Kernel& k, std::vector<bool>* tainted) {
     return T.ok;
 }
 
+static bool is_bid_x(const Node* n) {
+    while (n && n->kind == NK::Cast && n->kids.size() == 1) n = n->kids[0];
+    return n && n->kind == NK::Builtin && n->ref == 3;
+}
+static bool stores_bid_private(const Kernel& k, const Stmt* s) {
+    if (!s) return true;
+    if (s->kind == SK::Store && s->arr >= 0 && k.arrays[(size_t)s->arr].space == GLOBAL)
+        if (s->index.size() != 1 || !is_bid_x(s->index[0])) return false;
+    for (const Stmt* c : s->seq)
+        if (!stores_bid_private(k, c)) return false;
+    return stores_bid_private(k, s->body) && stores_bid_private(k, s->other) && stores_bid_private(k, s->init) &&
+           stores_bid_private(k, s->step);
+}
+bool block_private_outputs(const Kernel& k) {
+    for (const ArrayDecl& a : k.arrays)
+        if (a.space == GLOBAL && a.written && a.read) return false;
+    return stores_bid_private(k, k.body);
+}
+
 std::string generate_cuda(const Kernel& k, const CodegenOptions& opt) {
     Gen g(k, opt);
     return g.run();

@@ -805,7 +805,7 @@ __device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 // arena only (K1 initialises them there only, K2b flags the whole group)
 template <int A>
 __device__ __forceinline__ void pg_xb_mark_ms(const PgT& t, u32 flat) {
-    if (pg_sL.nblocks > 1u) {   // (the group's first arena: every seed touches the same cells; K2b
+    if (pg_sL.nblocks > 1u && PG_ARR(A).off_xf != ~0ull) {   // (the group's first arena: every seed touches the same cells; K2b
                                 //  decides for the whole group)
         atomicMin(t.arena + PG_ARR(A).off_xf + flat, t.blk + 1u);
         atomicMax(t.arena + PG_ARR(A).off_xl + flat, t.blk + 1u);
@@ -1008,7 +1008,7 @@ __device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
 }
 template <int A>
 __device__ __forceinline__ void pg_xb_mark_ms(const PgT& t, u32 flat) {
-    if (pg_sL.nblocks > 1u) {   // (the group's first arena: every seed touches the same cells; K2b
+    if (pg_sL.nblocks > 1u && PG_ARR(A).off_xf != ~0ull) {   // (the group's first arena: every seed touches the same cells; K2b
                                 //  decides for the whole group)
         atomicMin(t.arena + PG_ARR(A).off_xf + flat, t.blk + 1u);
         atomicMax(t.arena + PG_ARR(A).off_xl + flat, t.blk + 1u);
@@ -1167,7 +1167,7 @@ __device__ __forceinline__ void pg_check_gt_ms(const PgC& C, PgT& t, PgCold& c, 
 // block-parallel pass must be redone sequentially).
 template <int A>
 __device__ __forceinline__ void pg_xb_mark(const PgT& t, u32 flat) {
-    if (pg_sL.nblocks > 1u) {
+    if (pg_sL.nblocks > 1u && PG_ARR(A).off_xf != ~0ull) {   // (~0: block-private outputs, no XB)
         atomicMin(t.arena + PG_ARR(A).off_xf + flat, t.blk + 1u);
         atomicMax(t.arena + PG_ARR(A).off_xl + flat, t.blk + 1u);
     }

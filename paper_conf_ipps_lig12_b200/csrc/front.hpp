@@ -140,4 +140,12 @@ std::string generate_cuda(const Kernel& k, const CodegenOptions& opt);
 // tainted[v]: variable v may hold an input-dependent value (one copy per seed).
 bool seed_oblivious(const Kernel& k, std::vector<bool>* tainted = nullptr);
 
+// Block-private outputs: every global array the kernel writes is never loaded and every store
+// to it has the flat index `bid.x` (casts aside).  Blocks with distinct bid.x then write
+// distinct cells and read none that another block writes, so with a one-dimensional grid
+// (and gdim.x <= 2^bits, the index being w-bit arithmetic, X23) no global cell is shared
+// between blocks (X4 XB cannot occur): the planner drops the XB stamps and K2b for such
+// launches.  The SDK reductions' `g_odata[bid.x] = sdata[0]` is the case it is for.
+bool block_private_outputs(const Kernel& k);
+
 }  // namespace pgf

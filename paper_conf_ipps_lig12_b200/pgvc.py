@@ -78,7 +78,7 @@ class PgError(RuntimeError):
 _lib = None
 EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_equiv_seq", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
            "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_collect_vcliteral", "pg_ir_info",
-           "pg_ir_seed_oblivious",
+           "pg_ir_seed_oblivious", "pg_ir_block_private",
            "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals", "pg_merge_counters",
            "pg_measure_int32_peak",
            "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
@@ -115,6 +115,7 @@ def lib():
     L.pg_ir_info.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32),
                              ctypes.POINTER(ctypes.c_uint32)]
     L.pg_ir_seed_oblivious.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32)]
+    L.pg_ir_block_private.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32)]
     L.pg_ir_source.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_char_p,
                                ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]
     L.pg_ir_compile.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32]
@@ -131,7 +132,7 @@ def lib():
     for f in ("pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_equiv_seq", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
               "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_collect_vcliteral",
               "pg_ir_info",
-              "pg_ir_seed_oblivious", "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals",
+              "pg_ir_seed_oblivious", "pg_ir_block_private", "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals",
               "pg_merge_counters", "pg_measure_int32_peak"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
@@ -166,6 +167,12 @@ class Ir:
         o, n = ctypes.c_uint32(), ctypes.c_uint32()
         _ck(lib().pg_ir_seed_oblivious(self._h, ctypes.byref(o), ctypes.byref(n)))
         return bool(o.value), n.value
+
+    def block_private(self) -> bool:
+        """pg_ir_block_private: every written global array is write-only at index bid.x."""
+        b = ctypes.c_uint32()
+        _ck(lib().pg_ir_block_private(self._h, ctypes.byref(b)))
+        return bool(b.value)
 
     def source(self, bits=32, checks=CHK_RACE | CHK_OOB, bank_model=0) -> str:
         n = ctypes.c_size_t()

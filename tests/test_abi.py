@@ -136,6 +136,35 @@ def test_seed_oblivious_cases(pgvc, body, oblivious):
     assert pgvc.load_ir(text).seed_oblivious()[0] == oblivious
 
 
+def test_block_private_subjects(pgvc, W):
+    """The SDK reductions write g_odata[bid.x] only (never read): no cell can be shared
+    between blocks of a 1-D grid.  The transposes, scans, matmuls and bitonic sorts write
+    at thread-dependent indices; the two-pass reduction reads what it writes."""
+    subj = sorted(f[:-4] for f in os.listdir(os.path.join(ROOT, "subjects")) if f.endswith(".pgk"))
+    private = {n for n in subj if pgvc.load_ir(W.subject(n)).block_private()}
+    assert {"reduce0", "reduce1", "reduce2", "reduce2_obo", "reduce3", "reduce4", "reduce5", "reduce6"} <= private
+    for n in ("naive_transpose", "optimized_transpose", "prescan", "prescan_padded", "matmul_naive",
+              "matmul_tiled", "bitonic_global", "bitonic_shared"):
+        assert n not in private, n
+
+
+@pytest.mark.parametrize("stores,private", [
+    ("b[bid.x] = a[tid.x];", True),
+    ("if (tid.x == 0) b[(unsigned)bid.x] = 1;", True),
+    ("b[bid.x] = 1; b[bid.x] = 2;", True),
+    ("b[bid.x + 1] = 1;", False),                  # two blocks can meet on a cell
+    ("b[bid.y] = 1;", False),                      # only bid.x is analysed
+    ("b[tid.x] = 1;", False),
+    ("b[bid.x] = b[bid.x] + 1;", False),           # the output is read
+    ("unsigned i = bid.x; b[i] = 1;", False),      # (the index must be bid.x itself)
+    ("a[bid.x] = 1;", False),                      # a is read below
+])
+def test_block_private_cases(pgvc, stores, private):
+    text = ("kernel k(global inout int a[n], global out int b[n], unsigned n) {\n"
+            "  int x = a[tid.x];\n  %s\n}\n" % stores)
+    assert pgvc.load_ir(text).block_private() == private
+
+
 @pytest.mark.parametrize("body,checked,elided", [
     # the back-edge follows the body's last barrier: the first back-edge of its round
     ("for (int i = 0; i < n; i++) { s[tid.x] = i; sync; }", 0, 1),

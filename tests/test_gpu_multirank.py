@@ -112,6 +112,7 @@ def _bench_contract(d):
     assert abs(r["achieved"] * 1e12 - achieved) <= 1e-6 * achieved
     assert abs(r["frac"] - r["achieved"] / r["peak"]) <= 1e-9
     assert 0 < r["frac"] < 1 and 0 < r["frac_counted_ops"] < r["frac"]
+    assert abs(r["frac_of_both_pipes"] - r["achieved"] / r["peak_both_pipes"]) <= 1e-9
     assert r["k2_busy_ms_per_step"] <= d["ms_per_step"] * 1.0001
     assert d["gpu_launches"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert d["step_ms"]["min"] <= d["step_ms"]["median"] <= d["step_ms"]["max"]
