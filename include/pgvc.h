@@ -237,6 +237,12 @@ int pg_ir_seed_oblivious(const pg_ir *k, uint32_t *oblivious, uint32_t *n_tainte
  * cannot occur and checks of such launches skip the XB stamps, K2b and the sequential pass
  * (the SDK reductions' g_odata[bid.x]).  PG_E_ARG on a null kernel. */
 int pg_ir_block_private(const pg_ir *k, uint32_t *block_private);
+/* *mask bit a (arrays in declaration order) = 1 when array a is a one-dimensional shared
+ * array every store of which has the flat index tid.x (or a variable only ever assigned
+ * tid.x): in a one-dimensional block no two threads store to one cell, so no WW race on it
+ * is possible and its stores take a plain owner stamp instead of a claim (
+ * the SDK reductions' sdata[tid]).  PG_E_ARG on a null kernel. */
+int pg_ir_thread_private(const pg_ir *k, uint64_t *mask);
 /* Generated CUDA source of the evaluation kernel for (bits, checks, bank_model). */
 int pg_ir_source(const pg_ir *k, uint32_t bits, uint32_t checks, uint32_t bank_model, char *buf, size_t cap,
                  size_t *len);

@@ -871,6 +871,100 @@ bool block_private_outputs(const Kernel& k) {
     return stores_bid_private(k, k.body);
 }
 
+static const Node* strip_casts(const Node* n) {
+    while (n && n->kind == NK::Cast && n->kids.size() == 1) n = n->kids[0];
+    return n;
+}
+static bool is_tid_x(const Node* n) {
+    n = strip_casts(n);
+    return n && n->kind == NK::Builtin && n->ref == 0;
+}
+static void count_assigns(const Stmt* s, std::vector<int>& n) {
+    if (!s) return;
+    if (s->kind == SK::Assign && s->var >= 0) n[(size_t)s->var]++;
+    for (const Stmt* c : s->seq) count_assigns(c, n);
+    count_assigns(s->body, n);
+    count_assigns(s->other, n);
+    count_assigns(s->init, n);
+    count_assigns(s->step, n);
+}
+static bool node_mentions(const Node* e, int v) {
+    if (!e) return false;
+    if (e->kind == NK::Var && e->ref == v) return true;
+    for (const Node* c : e->kids)
+        if (node_mentions(c, v)) return true;
+    return false;
+}
+static bool stmt_mentions(const Stmt* s, int v) {
+    if (!s) return false;
+    if (s->kind == SK::Assign && s->var == v) return true;
+    if (node_mentions(s->value, v) || node_mentions(s->cond, v)) return true;
+    for (const Node* i : s->index)
+        if (node_mentions(i, v)) return true;
+    for (const Stmt* c : s->seq)
+        if (stmt_mentions(c, v)) return true;
+    return stmt_mentions(s->body, v) || stmt_mentions(s->other, v) || stmt_mentions(s->init, v) ||
+           stmt_mentions(s->step, v);
+}
+struct TpCtx {
+    const Kernel& k;
+    std::vector<int> nassign;
+    std::vector<bool> alias;   // top-level variables that hold tid.x wherever they are used
+    bool tid_value(const Node* v) const {
+        v = strip_casts(v);
+        return is_tid_x(v) || (v && v->kind == NK::Var && v->ref >= 0 && alias[(size_t)v->ref]);
+    }
+};
+// Store sites: index tid.x, a top-level alias, or the hidden copy a compound assignment
+// `s[t] op= e` makes of its index right before the store (X21: [h = t; s[h] = s[h] op e])
+static void tp_stores(const TpCtx& x, const Stmt* s, std::vector<bool>& tp) {
+    if (!s) return;
+    for (size_t p = 0; p < s->seq.size(); p++) {
+        const Stmt* c = s->seq[p];
+        if (c && c->kind == SK::Store && c->arr >= 0 && c->index.size() == 1) {
+            const Node* ix = strip_casts(c->index[0]);
+            if (!x.tid_value(ix) && ix && ix->kind == NK::Var && ix->ref >= 0 && p > 0) {
+                const Stmt* d = s->seq[p - 1];
+                const int h = ix->ref;
+                if (d && d->kind == SK::Assign && d->var == h && x.nassign[(size_t)h] == 1 && x.tid_value(d->value))
+                    continue;   // (the compound pattern: the store is fine)
+            }
+        }
+        tp_stores(x, c, tp);
+    }
+    if (s->kind == SK::Store && s->arr >= 0) {
+        if (!(s->index.size() == 1 && x.tid_value(s->index[0]))) tp[(size_t)s->arr] = false;
+    }
+    tp_stores(x, s->body, tp);
+    tp_stores(x, s->other, tp);
+    tp_stores(x, s->init, tp);
+    tp_stores(x, s->step, tp);
+}
+std::vector<bool> thread_private_stores(const Kernel& k) {
+    TpCtx x{k, std::vector<int>(k.vars.size(), 0), std::vector<bool>(k.vars.size(), false)};
+    count_assigns(k.body, x.nassign);
+    // top-level aliases: the variable's only assignment is a top-level `v = tid.x` (or `= u`,
+    // u an alias defined earlier) and no earlier top-level statement mentions v (before it,
+    // v holds its initial 0, X21)
+    std::vector<const Stmt*> top;
+    if (k.body && k.body->kind == SK::Seq) top.assign(k.body->seq.begin(), k.body->seq.end());
+    else if (k.body) top.push_back(k.body);
+    for (size_t i = 0; i < top.size(); i++) {
+        const Stmt* st = top[i];
+        if (!st || st->kind != SK::Assign || st->var < 0) continue;
+        const int v = st->var;
+        if (k.vars[(size_t)v].scalar || x.nassign[(size_t)v] != 1 || !x.tid_value(st->value)) continue;
+        bool early = false;
+        for (size_t j = 0; j < i && !early; j++) early = stmt_mentions(top[j], v);
+        if (!early) x.alias[(size_t)v] = true;
+    }
+    std::vector<bool> tp(k.arrays.size(), false);
+    for (size_t a = 0; a < k.arrays.size(); a++)
+        tp[a] = k.arrays[a].space == SHARED && k.arrays[a].dims.size() == 1 && k.arrays[a].written;
+    tp_stores(x, k.body, tp);
+    return tp;
+}
+
 std::string generate_cuda(const Kernel& k, const CodegenOptions& opt) {
     Gen g(k, opt);
     return g.run();

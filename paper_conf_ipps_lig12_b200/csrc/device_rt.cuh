@@ -445,6 +445,14 @@ __device__ __forceinline__ u32 pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell,
 #else
 #define PG_GSH(A) ((pg_sL.arr[A].flags >> 1) & 1u)
 #endif
+// Shared arrays whose stores are all at index tid.x in a one-dimensional block (PgArr flags
+// bit 2, PgSA::tp; pg_ir_thread_private): no two threads store to one cell, so no WW race
+// on them - stores take a plain owner stamp, no claim, and a check reads only reader stamps
+#ifdef PG_S_T
+#define PG_TP(A) ((u32)PgSA<A>::tp)
+#else
+#define PG_TP(A) ((pg_sL.arr[A].flags >> 2) & 1u)
+#endif
 template <int A> __device__ __forceinline__ u32* pg_gown(const PgT& t) {
     return PG_GSH(A) ? pg_sh(t, PG_SH(A, s_own)) : t.arena + PG_ARR(A).off_own;
 }
@@ -465,6 +473,7 @@ template <int A> __device__ __forceinline__ u32* pg_grmax(const PgT& t) {
 // during a round outside the data-flow dump.
 template <int A>
 __device__ __forceinline__ void pg_claim_sh(const PgC& C, const PgT& t, u32 flat) {
+    if (PG_TP(A)) return;   // (the writer owns the cell: the check commits it, no WW possible)
     atomicMin(pg_sh(t, PG_CAS ? PG_SH(A, s_clm) : PG_SH(A, s_own)) + flat, pg_stamp_min(C, t));
 #if PG_RACECHK
     if (PG_T > 1u) atomicMax(pg_sh(t, PG_SH(A, s_wmax)) + flat, pg_stamp_max(C, t));
@@ -662,13 +671,13 @@ template <int A, bool RDA>
 __device__ __forceinline__ void pg_commit_sh(const PgC& C, PgT& t, PgCold& c, u32 flat, u32 val) {
     u32* own = pg_sh(t, PG_SH(A, s_own)) + flat;
     const u32 me = C.smin | t.tlin;
-    if (PG_T > 1u) {
+    if (PG_T > 1u && !PG_TP(A)) {
         const u32 old = atomicMin(own, me);
         t.fl |= (old ^ me) - 1u < 0xFFFu;   // another writer's stamp of this round (WW)
-        if (RDA) pg_flog(t, c, ((u32)A << 24) | flat);
     } else {
-        *own = me;
+        *own = me;   // (one thread per block writes the cell: no claim)
     }
+    if (PG_T > 1u && RDA) pg_flog(t, c, ((u32)A << 24) | flat);
     pg_sh(t, PG_SH(A, s_val))[flat] = val;
     pg_fcount(t);
 }
@@ -790,13 +799,13 @@ __device__ __forceinline__ void pg_st_sh_ms(PgC& C, PgT& t, PgCold& c, u64* ss, 
     }
     u32* own = pg_sh(t, PG_SH(A, s_own)) + flat;
     const u32 me = C.smin | t.tlin;
-    if (PG_T > 1u) {
+    if (PG_T > 1u && !PG_TP(A)) {
         const u32 old = atomicMin(own, me);
         t.fl |= (old ^ me) - 1u < 0xFFFu;   // another writer's stamp of this round (WW)
-        if (RDA) pg_flog(t, c, ((u32)A << 24) | flat);
     } else {
-        *own = me;
+        *own = me;   // (one thread per block writes the cell: no claim)
     }
+    if (PG_T > 1u && RDA) pg_flog(t, c, ((u32)A << 24) | flat);
     pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, val);
     pg_fcount(t);
 }
@@ -1108,14 +1117,15 @@ __device__ __forceinline__ void pg_check_sh_ms(const PgC& C, PgT& t, PgCold& c, 
         pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
         return;
     }
-    const u32 own = pg_sh(t, PG_CAS ? PG_SH(A, s_clm) : PG_SH(A, s_own))[flat];
+    // (thread-private stores: the writer owns its cell, no claim was made)
+    const u32 own = PG_TP(A) ? pg_stamp_min(C, t) : pg_sh(t, PG_CAS ? PG_SH(A, s_clm) : PG_SH(A, s_own))[flat];
     if (own == pg_stamp_min(C, t)) {
         pg_vst(pg_sh(t, PG_SH(A, s_val)) + flat * PG_MS, v);
-        if (PG_CAS) pg_sh(t, PG_SH(A, s_own))[flat] = own;
+        if (PG_CAS || PG_TP(A)) pg_sh(t, PG_SH(A, s_own))[flat] = own;
     }
 #if PG_RACECHK
     if (PG_T > 1u) {
-        const u32 wmax = pg_sh(t, PG_SH(A, s_wmax))[flat];
+        const u32 wmax = PG_TP(A) ? pg_stamp_max(C, t) : pg_sh(t, PG_SH(A, s_wmax))[flat];
         const u32 rmin = RD ? pg_sh(t, PG_SH(A, s_rmin))[flat] : 0u;
         const u32 rmax = RD ? pg_sh(t, PG_SH(A, s_rmax))[flat] : 0u;
         if ((wmax & 0xFFFu) != (own & 0xFFFu) ||
@@ -1324,14 +1334,15 @@ __device__ __forceinline__ void pg_check_sh(const PgC& C, PgT& t, PgCold& c, u32
         pg_sh(t, PG_SH(A, s_val))[flat] = val;
         return;
     }
-    const u32 own = pg_sh(t, PG_CAS ? PG_SH(A, s_clm) : PG_SH(A, s_own))[flat];
+    // (thread-private stores: the writer owns its cell, no claim was made)
+    const u32 own = PG_TP(A) ? pg_stamp_min(C, t) : pg_sh(t, PG_CAS ? PG_SH(A, s_clm) : PG_SH(A, s_own))[flat];
     if (own == pg_stamp_min(C, t)) {
         pg_sh(t, PG_SH(A, s_val))[flat] = val;
-        if (PG_CAS) pg_sh(t, PG_SH(A, s_own))[flat] = own;
+        if (PG_CAS || PG_TP(A)) pg_sh(t, PG_SH(A, s_own))[flat] = own;
     }
 #if PG_RACECHK
     if (PG_T > 1u) {
-        const u32 wmax = pg_sh(t, PG_SH(A, s_wmax))[flat];
+        const u32 wmax = PG_TP(A) ? pg_stamp_max(C, t) : pg_sh(t, PG_SH(A, s_wmax))[flat];
         const u32 rmin = RD ? pg_sh(t, PG_SH(A, s_rmin))[flat] : 0u;
         const u32 rmax = RD ? pg_sh(t, PG_SH(A, s_rmax))[flat] : 0u;
         // (a cell only its writer read this round is no RW race: skip the slow path)

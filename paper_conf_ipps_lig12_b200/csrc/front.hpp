@@ -148,4 +148,12 @@ bool seed_oblivious(const Kernel& k, std::vector<bool>* tainted = nullptr);
 // launches.  The SDK reductions' `g_odata[bid.x] = sdata[0]` is the case it is for.
 bool block_private_outputs(const Kernel& k);
 
+// Thread-private stores: for each array, true when it is a one-dimensional shared array and
+// every store to it has the flat index tid.x (or a variable whose every assignment is tid.x;
+// casts aside).  With a one-dimensional block, two threads of a block then never store to one
+// cell: no WW race on it is possible, so its stores need no ownership claim (a plain owner
+// stamp), and a check needs only its reader stamps (device_rt PG_TP; the SDK reductions'
+// `sdata[tid] += sdata[tid + s]`).
+std::vector<bool> thread_private_stores(const Kernel& k);
+
 }  // namespace pgf

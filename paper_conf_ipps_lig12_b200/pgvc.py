@@ -78,7 +78,7 @@ class PgError(RuntimeError):
 _lib = None
 EXPORTS = ["pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_equiv_seq", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
            "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_collect_vcliteral", "pg_ir_info",
-           "pg_ir_seed_oblivious", "pg_ir_block_private",
+           "pg_ir_seed_oblivious", "pg_ir_block_private", "pg_ir_thread_private",
            "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals", "pg_merge_counters",
            "pg_measure_int32_peak",
            "pg_last_error", "pg_ir_free", "pg_run_free", "pg_version"]
@@ -116,6 +116,7 @@ def lib():
                              ctypes.POINTER(ctypes.c_uint32)]
     L.pg_ir_seed_oblivious.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32)]
     L.pg_ir_block_private.argtypes = [vp, ctypes.POINTER(ctypes.c_uint32)]
+    L.pg_ir_thread_private.argtypes = [vp, ctypes.POINTER(ctypes.c_uint64)]
     L.pg_ir_source.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_char_p,
                                ctypes.c_size_t, ctypes.POINTER(ctypes.c_size_t)]
     L.pg_ir_compile.argtypes = [vp, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32]
@@ -132,7 +133,7 @@ def lib():
     for f in ("pg_load_ir", "pg_check_equiv", "pg_check_equiv_n", "pg_check_equiv_seq", "pg_check_races", "pg_check_banks", "pg_check_property", "pg_collect_cex",
               "pg_collect_site_stats", "pg_collect_dataflow", "pg_collect_lockstep", "pg_collect_vcliteral",
               "pg_ir_info",
-              "pg_ir_seed_oblivious", "pg_ir_block_private", "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals",
+              "pg_ir_seed_oblivious", "pg_ir_block_private", "pg_ir_thread_private", "pg_ir_source", "pg_ir_compile", "pg_run_timing", "pg_run_intervals",
               "pg_merge_counters", "pg_measure_int32_peak"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
@@ -173,6 +174,12 @@ class Ir:
         b = ctypes.c_uint32()
         _ck(lib().pg_ir_block_private(self._h, ctypes.byref(b)))
         return bool(b.value)
+
+    def thread_private(self) -> int:
+        """pg_ir_thread_private: bit a = array a's stores are all at index tid.x."""
+        m = ctypes.c_uint64()
+        _ck(lib().pg_ir_thread_private(self._h, ctypes.byref(m)))
+        return m.value
 
     def source(self, bits=32, checks=CHK_RACE | CHK_OOB, bank_model=0) -> str:
         n = ctypes.c_size_t()

@@ -165,6 +165,36 @@ def test_block_private_cases(pgvc, stores, private):
     assert pgvc.load_ir(text).block_private() == private
 
 
+def test_thread_private_subjects(pgvc, W):
+    """sdata[tid] (reduce0, reduce3..6) and sdata[t] with t = tid.x (reduce2 and its off-by-one
+    mutant) are thread-private stores; reduce1's sdata[2 s tid], the scans' temp[ai] and the
+    transposes' 2-D tile are not."""
+    def tp(name):
+        return pgvc.load_ir(W.subject(name)).thread_private()
+    for n in ("reduce0", "reduce2", "reduce2_obo", "reduce3", "reduce4", "reduce5", "reduce6"):
+        assert tp(n) != 0, n
+    for n in ("reduce1", "prescan", "prescan_padded", "optimized_transpose", "bitonic_shared", "matmul_tiled"):
+        assert tp(n) == 0, n
+
+
+@pytest.mark.parametrize("body,private", [
+    ("s[tid.x] = a[tid.x];", True),
+    ("unsigned t = tid.x; s[t] = 1; s[t] = s[t] + a[t];", True),
+    ("unsigned t = tid.x; t = t + 1; s[t] = 1;", False),    # t is not tid.x throughout
+    ("s[tid.x + 1] = 1;", False),
+    ("s[tid.y] = 1;", False),
+    ("if (tid.x == 0) s[0] = 1;", False),
+    ("s[(unsigned)tid.x] = 2;", True),
+    ("unsigned t = tid.x; s[t] += a[t];", True),            # compound: s[h] with h = t (X21)
+    ("unsigned t; s[t] = 1; t = tid.x;", False),            # t is 0 at the store (X21)
+    ("unsigned u; unsigned v = u; u = v; s[v] = 1;", False),  # no tid.x at the root
+    ("unsigned t = tid.x; if (t < 4u) t = 0; s[t] = 1;", False),
+])
+def test_thread_private_cases(pgvc, body, private):
+    text = ("kernel k(global in int a[n], unsigned n) {\n  shared int s[bdim.x];\n  %s\n}\n" % body)
+    assert bool((pgvc.load_ir(text).thread_private() >> 1) & 1) == private    # s is array 1 (a is array 0)
+
+
 @pytest.mark.parametrize("body,checked,elided", [
     # the back-edge follows the body's last barrier: the first back-edge of its round
     ("for (int i = 0; i < n; i++) { s[tid.x] = i; sync; }", 0, 1),

@@ -5,6 +5,8 @@
   a read-and-written global array with races, in one block (promoted) and in four (arena);
 * the streamed comparison (K3) on array sizes that are not multiples of its 4-cell loads;
 * alternating input definitions (RAND32 / RANGE) on one launch list: one plan each.
+* thread-private shared stores (PgArr flags bit 2: stores at s[tid.x] in a 1-D block take no
+  claim) with RW races, and the same kernels in 2-D blocks, where the stores collide (WW).
 The fixtures are small kernels written for these paths (X4 races, X16 records)."""
 import pytest
 
@@ -122,3 +124,56 @@ def test_alternating_input_definitions(env, oracle, W):  # noqa: F811
         ref, recs, summ, _ = run_pair(env, oracle, W.subject(w.src), W.subject(w.tgt), w.launch_src, w.launch_tgt,
                                       n_seeds=3, input_mode=mode, input_range=rng)
         assert_same(ref, recs, summ)
+
+
+# thread-private stores (every store at s[t], t = tid.x): RW races between neighbours, a
+# thread storing twice in a round, compound stores; in a 2-D block the same stores collide
+# (tid.x repeats across tid.y), so the WW races there must still be found (no PG_TP)
+TP_RACY = """
+kernel tp_racy(global in int x[n], global out int y[n], unsigned n) {
+  shared int s[bdim.x];
+  unsigned t = tid.x;
+  unsigned i = (bid.x * bdim.y + tid.y) * bdim.x + t;
+  s[t] = (i < n) ? x[i] : 0;
+  sync;
+  if (t + 1 < bdim.x) s[t] += s[t + 1];
+  s[t] = s[t] + tid.y;
+  sync;
+  if (i < n) y[i] = s[(t * 3u) % bdim.x];
+}
+"""
+TP_CLEAN = """
+kernel tp_clean(global in int x[n], global out int y[n], unsigned n) {
+  shared int s[bdim.x];
+  unsigned t = tid.x;
+  unsigned i = (bid.x * bdim.y + tid.y) * bdim.x + t;
+  s[t] = (i < n) ? x[i] : 0;
+  sync;
+  int v = s[t];
+  if (t + 1 < bdim.x) v = v + s[t + 1];
+  sync;
+  s[t] = v + tid.y;
+  sync;
+  if (i < n) y[i] = s[(t * 3u) % bdim.x];
+}
+"""
+
+
+@pytest.mark.parametrize("seeds", [1, 9])
+def test_thread_private_stores(env, oracle, W, seeds):  # noqa: F811
+    pgvc, _ = env
+    assert pgvc.load_ir(TP_RACY).thread_private() == 0b100 == pgvc.load_ir(TP_CLEAN).thread_private()
+    ls = [W.Launch((g, 1, 1), (b, 1, 1), (g * b,)) for b in (1, 2, 5, 32, 64, 256, 1024) for g in (1, 3)]
+    ref, recs, summ, _ = run_pair(env, oracle, TP_RACY, TP_CLEAN, ls, n_seeds=seeds)
+    assert_same(ref, recs, summ)
+    assert summ["per_kind"][3] > 0      # RW races found (X16 kind order: ..., RACE_RW)
+
+
+def test_thread_private_stores_in_2d_blocks_still_race(env, oracle, W):  # noqa: F811
+    ls = [W.Launch((g, 1, 1), (bx, by, 1), (g * bx * by,)) for (bx, by) in ((2, 2), (4, 8), (32, 4), (1, 3))
+          for g in (1, 2)]
+    ref, recs, summ, _ = run_pair(env, oracle, TP_RACY, TP_CLEAN, ls, n_seeds=3)
+    assert_same(ref, recs, summ)
+    ref, recs, summ, _ = run_pair(env, oracle, TP_CLEAN, None, ls, mode=1, n_seeds=3)
+    assert_same(ref, recs, summ)
+    assert summ["n_fail"] > 0           # s[tid.x] from several tid.y: WW
