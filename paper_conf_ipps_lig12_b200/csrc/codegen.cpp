@@ -265,6 +265,20 @@ struct Gen {
 
     Gen(const Kernel& k, const CodegenOptions& o) : K(k), O(o) {
         mask = o.bits >= 32 ? 0xFFFFFFFFu : ((1u << o.bits) - 1u);
+        tidv_ = tid_alias_vars(k);
+        tpa_ = thread_private_stores(k);
+    }
+    // optimistic pass: a load of a thread-private array at index tid.x reads the cell only its
+    // own thread writes - it cannot be half of a RW race, so (when the launch's block is 1-D,
+    // PgSA::tp) it takes no reader stamp.  The exact protocol keeps every reader stamp: X16's
+    // RW record takes the minimum / maximum reader over all of them.
+    std::vector<bool> tidv_, tpa_;
+    bool self_load(const Node* n) const {
+        if (!O.fast || n->kids.size() != 1 || !tpa_[(size_t)n->ref]) return false;
+        const Node* ix = n->kids[0];
+        while (ix && ix->kind == NK::Cast && ix->kids.size() == 1) ix = ix->kids[0];
+        return ix && ((ix->kind == NK::Builtin && ix->ref == 0) ||
+                      (ix->kind == NK::Var && ix->ref >= 0 && tidv_[(size_t)ix->ref]));
     }
 
     std::string tmp(const char* p = "t") { return std::string("_") + p + std::to_string(ntmp++); }
@@ -357,7 +371,8 @@ struct Gen {
             std::string f = flat_index(n, n->ref, pr);
             std::string r = tmp();
             std::string A = std::to_string(n->ref), S = std::to_string(n->site) + "u";
-            const std::string st = stamps_needed(n) ? "true" : "false", lg = log_[(size_t)n->ref] ? "true" : "false";
+            const std::string st = !stamps_needed(n) ? "false" : self_load(n) ? "!PG_TP_CONST(" + A + ")" : "true";
+            const std::string lg = log_[(size_t)n->ref] ? "true" : "false";
             if (ms()) {   // (seed-oblivious: shared or global, never private)
                 line("u32 " + r + "[PG_MS];");
                 tnames_.insert(r);
@@ -940,7 +955,31 @@ static void tp_stores(const TpCtx& x, const Stmt* s, std::vector<bool>& tp) {
     tp_stores(x, s->init, tp);
     tp_stores(x, s->step, tp);
 }
-std::vector<bool> thread_private_stores(const Kernel& k) {
+static TpCtx tp_ctx(const Kernel& k);
+std::vector<bool> tid_alias_vars(const Kernel& k) {
+    TpCtx x = tp_ctx(k);
+    // plus the hidden copies compound stores make of their index (X21): assigned once, right
+    // before the store that reads and writes through them
+    std::vector<bool> out = x.alias;
+    struct W {
+        const TpCtx& x;
+        std::vector<bool>& out;
+        void go(const Stmt* s) {
+            if (!s) return;
+            if (s->kind == SK::Assign && s->var >= 0 && x.k.vars[(size_t)s->var].hidden &&
+                x.nassign[(size_t)s->var] == 1 && x.tid_value(s->value))
+                out[(size_t)s->var] = true;
+            for (const Stmt* c : s->seq) go(c);
+            go(s->body);
+            go(s->other);
+            go(s->init);
+            go(s->step);
+        }
+    } w{x, out};
+    w.go(k.body);
+    return out;
+}
+static TpCtx tp_ctx(const Kernel& k) {
     TpCtx x{k, std::vector<int>(k.vars.size(), 0), std::vector<bool>(k.vars.size(), false)};
     count_assigns(k.body, x.nassign);
     // top-level aliases: the variable's only assignment is a top-level `v = tid.x` (or `= u`,
@@ -958,6 +997,10 @@ std::vector<bool> thread_private_stores(const Kernel& k) {
         for (size_t j = 0; j < i && !early; j++) early = stmt_mentions(top[j], v);
         if (!early) x.alias[(size_t)v] = true;
     }
+    return x;
+}
+std::vector<bool> thread_private_stores(const Kernel& k) {
+    TpCtx x = tp_ctx(k);
     std::vector<bool> tp(k.arrays.size(), false);
     for (size_t a = 0; a < k.arrays.size(); a++)
         tp[a] = k.arrays[a].space == SHARED && k.arrays[a].dims.size() == 1 && k.arrays[a].written;

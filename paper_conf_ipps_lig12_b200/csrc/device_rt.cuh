@@ -450,8 +450,10 @@ __device__ __forceinline__ u32 pg_log_write(PgC& C, PgT& t, PgCold& c, u32 cell,
 // on them - stores take a plain owner stamp, no claim, and a check reads only reader stamps
 #ifdef PG_S_T
 #define PG_TP(A) ((u32)PgSA<A>::tp)
+#define PG_TP_CONST(A) (PgSA<A>::tp != 0u)   // (a template argument: shape variants only)
 #else
 #define PG_TP(A) ((pg_sL.arr[A].flags >> 2) & 1u)
+#define PG_TP_CONST(A) false
 #endif
 template <int A> __device__ __forceinline__ u32* pg_gown(const PgT& t) {
     return PG_GSH(A) ? pg_sh(t, PG_SH(A, s_own)) : t.arena + PG_ARR(A).off_own;

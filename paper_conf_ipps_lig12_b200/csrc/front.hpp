@@ -155,5 +155,8 @@ bool block_private_outputs(const Kernel& k);
 // stamp), and a check needs only its reader stamps (device_rt PG_TP; the SDK reductions'
 // `sdata[tid] += sdata[tid + s]`).
 std::vector<bool> thread_private_stores(const Kernel& k);
+// Variables holding tid.x wherever they are read: top-level aliases (thread_private_stores)
+// and the hidden copies compound stores make of their index (X21).
+std::vector<bool> tid_alias_vars(const Kernel& k);
 
 }  // namespace pgf

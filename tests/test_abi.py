@@ -177,6 +177,18 @@ def test_thread_private_subjects(pgvc, W):
         assert tp(n) == 0, n
 
 
+def test_self_loads_skip_reader_stamps_in_the_optimistic_pass(pgvc, W):
+    """reduce2's `sdata[t] += sdata[t + s]`: the load of the thread's own cell (through the
+    compound store's index copy, X21) can skip its reader stamp in the optimistic pass when the
+    block is 1-D (PgSA::tp); the load of sdata[t + s] keeps it; the exact pass keeps both."""
+    k = pgvc.load_ir(W.subject("reduce2"))
+    fast = [l for l in k.source(checks=pgvc.CHK_RACE | pgvc.CHK_OOB | (1 << 30)).split("\n") if "pg_ld_sh<" in l]
+    exact = [l for l in k.source(checks=pgvc.CHK_RACE | pgvc.CHK_OOB).split("\n") if "pg_ld_sh<" in l]
+    assert any("!PG_TP_CONST(2)" in l and ", 3u)" in l for l in fast)      # site 3: sdata[t] (read)
+    assert any("<2, true," in l and ", 5u)" in l for l in fast)            # site 5: sdata[t + s]
+    assert not any("PG_TP_CONST" in l for l in exact)
+
+
 @pytest.mark.parametrize("body,private", [
     ("s[tid.x] = a[tid.x];", True),
     ("unsigned t = tid.x; s[t] = 1; s[t] = s[t] + a[t];", True),
