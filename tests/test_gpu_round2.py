@@ -177,3 +177,20 @@ def test_thread_private_stores_in_2d_blocks_still_race(env, oracle, W):  # noqa:
     ref, recs, summ, _ = run_pair(env, oracle, TP_CLEAN, None, ls, mode=1, n_seeds=3)
     assert_same(ref, recs, summ)
     assert summ["n_fail"] > 0           # s[tid.x] from several tid.y: WW
+
+
+@pytest.mark.parametrize("bits", [8, 12])
+def test_narrow_widths_keep_xb_and_ww(env, oracle, W, bits):  # noqa: F811
+    # w-bit index arithmetic (X23): at 8 bits tid.x and bid.x wrap at 256, so blocks of 512
+    # threads store sdata[tid] to one cell twice (WW) and grids of 512 blocks store
+    # g_odata[bid.x] to one cell twice (XB): neither the thread-private nor the
+    # block-private shortcut may apply there
+    ls, lt = [], []
+    for N, B in ((1024, 512), (1024, 2), (8192, 4), (4096, 1024)):
+        ls.append(W.reduce_launch("reduce0", N, B))
+        lt.append(W.reduce_launch("reduce2", N, B))
+    ref, recs, summ, _ = run_pair(env, oracle, W.subject("reduce0"), W.subject("reduce2"), ls, lt, n_seeds=3,
+                                  bits=bits)
+    assert_same(ref, recs, summ)
+    if bits == 8:
+        assert summ["per_kind"][2] > 0 and summ["per_kind"][4] > 0    # RACE_WW and RACE_XB
