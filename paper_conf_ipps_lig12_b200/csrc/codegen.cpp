@@ -757,6 +757,8 @@ struct Gen {
         o << "#define PG_LOCKSTEP " << ((O.checks & 64) ? 1 : 0) << "\n";
         o << "#define PG_FAST " << (O.fast ? 1 : 0) << "\n";
         // (store-time claims: not with bank / coalescing statistics, nor with PGVC_CAS=0 - api.cpp cas_on)
+        if (std::getenv("PGVC_PACK_OLD"))   // (diagnostics: round 1's 16/10/26/12 event prefix)
+            o << "#define PG_PACK_B0 16u\n#define PG_PACK_B1 10u\n#define PG_PACK_B2 26u\n#define PG_PACK_B3 12u\n";
         if (std::getenv("PGVC_RC_INLINE") && std::string(std::getenv("PGVC_RC_INLINE")) == "1")
             o << "#define PG_RC_INLINE __forceinline__\n";
         o << "#define PG_CAS_ON "

@@ -220,13 +220,21 @@ __device__ __forceinline__ bool pg_lex_less(const u32* a, const u32* b) {
     return false;
 }
 
-// Monotone 64-bit prefix of the X16 event order: (round, array, addr, tid_a) in 16 / 10 / 26 /
-// 12 bits, a field that does not fit saturates and zeroes the rest, so a <lex b implies
+// Monotone 64-bit prefix of the X16 event order: (round, array, addr, tid_a) in 16 / 10 / 24 /
+// 14 bits (in-bounds addresses are < 2^24, X5; tid_a is a global thread id, so the wider
+// field separates the events of more blocks before the lexicographic fallback), a field
+// that does not fit saturates and zeroes the rest, so a <lex b implies
 // pg_pack(a) <= pg_pack(b).  Slots keep ~pg_pack of their minimum (atomicMax): a candidate
 // whose pack is larger cannot be the minimum and skips the lock - thousands of CTAs that
 // report events of one instance (one slot) no longer serialise on it.
+#ifndef PG_PACK_B2
+#define PG_PACK_B0 16u
+#define PG_PACK_B1 10u
+#define PG_PACK_B2 24u
+#define PG_PACK_B3 14u
+#endif
 __device__ __forceinline__ u64 pg_pack(const u32* f) {
-    const u32 bits[4] = {16u, 10u, 26u, 12u};
+    const u32 bits[4] = {PG_PACK_B0, PG_PACK_B1, PG_PACK_B2, PG_PACK_B3};
     u64 k = 0;
     bool sat = false;
 #pragma unroll
